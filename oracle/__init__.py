@@ -1,0 +1,156 @@
+"""CPU oracle (TEST INFRASTRUCTURE ONLY).
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl reference legs may
+import this package.  It wraps the plain-C loop nest in ft_oracle.c (the paper's definitions,
+see that file's header for the PAPER.md citations) through ctypes.  It shares no code with the
+CUDA path (paper_conf_sosp_liuqc0hs0y24_b200/) and never imports it.
+
+Pins: tests/test_oracle_pins.py (P1–P12 of SURVEY.md §8(c) c.6).  The grid cell (R12–R14)
+is "parity unpinned" by the paper beyond its Ly=1 / Lx=1 reductions (P8).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "liboracle.so")
+_SOURCES = [os.path.join(_HERE, "ft_oracle.c"), os.path.join(_HERE, "ft_oracle_impl.h")]
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (-O2 -fopenmp; no -ffast-math: IEEE semantics kept)."""
+    newest = max(os.path.getmtime(s) for s in _SOURCES)
+    if not force and os.path.exists(LIB_PATH) and os.path.getmtime(LIB_PATH) >= newest:
+        return LIB_PATH
+    cmd = ["gcc", "-O2", "-march=x86-64-v2", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+           "-fvisibility=hidden", "-ffp-contract=off", "-o", LIB_PATH + ".tmp", _SOURCES[0], "-lm"]
+    subprocess.check_call(cmd, cwd=_HERE)
+    os.replace(LIB_PATH + ".tmp", LIB_PATH)
+    return LIB_PATH
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        _lib = ctypes.CDLL(LIB_PATH)
+        for sfx in ("f64", "f32"):
+            for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell"):
+                fn = getattr(_lib, f"ft_oracle_{name}_{sfx}")
+                fn.restype = ctypes.c_int if name != "lstm_cell" else None
+    return _lib
+
+
+def num_threads() -> int:
+    return int(lib().ft_oracle_num_threads())
+
+
+def _p(a):
+    return None if a is None else a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _prec(precision):
+    if precision == "f64":
+        return np.float64
+    if precision == "f32":
+        return np.float32
+    raise ValueError(precision)
+
+
+def _c(a, dt):
+    return np.ascontiguousarray(a, dtype=dt)
+
+
+def stacked_lstm(x, W, U, b, precision="f64", want_all=False):
+    """Stacked LSTM oracle (Listing 2).  x [B][T][H], W/U [D][4][H][H], b [D][4][H]."""
+    dt = _prec(precision)
+    B, T, H = x.shape
+    D = W.shape[0]
+    x, W, U, b = (_c(a, dt) for a in (x, W, U, b))
+    y = np.empty((B, T, H), dt)
+    h_n = np.empty((B, D, H), dt)
+    c_n = np.empty((B, D, H), dt)
+    h_all = np.empty((B, D, T, H), dt) if want_all else None
+    c_all = np.empty((B, D, T, H), dt) if want_all else None
+    rc = getattr(lib(), f"ft_oracle_stacked_lstm_{precision}")(
+        B, T, H, D, _p(x), _p(W), _p(U), _p(b), _p(y), _p(h_n), _p(c_n), _p(h_all), _p(c_all))
+    if rc:
+        raise RuntimeError(f"oracle stacked_lstm failed: {rc}")
+    out = dict(y=y, h_n=h_n, c_n=c_n)
+    if want_all:
+        out.update(h_all=h_all, c_all=c_all)
+    return out
+
+
+def dilated_rnn(x, W, U, b, dilations, precision="f64", want_all=False):
+    dt = _prec(precision)
+    B, T, H = x.shape
+    D = W.shape[0]
+    dil = np.ascontiguousarray(dilations, dtype=np.int32)
+    assert dil.shape == (D,)
+    x, W, U, b = (_c(a, dt) for a in (x, W, U, b))
+    y = np.empty((B, T, H), dt)
+    h_n = np.empty((B, D, H), dt)
+    c_n = np.empty((B, D, H), dt)
+    h_all = np.empty((B, D, T, H), dt) if want_all else None
+    c_all = np.empty((B, D, T, H), dt) if want_all else None
+    rc = getattr(lib(), f"ft_oracle_dilated_rnn_{precision}")(
+        B, T, H, D, _p(dil), _p(x), _p(W), _p(U), _p(b), _p(y), _p(h_n), _p(c_n),
+        _p(h_all), _p(c_all))
+    if rc:
+        raise RuntimeError(f"oracle dilated_rnn failed: {rc}")
+    out = dict(y=y, h_n=h_n, c_n=c_n)
+    if want_all:
+        out.update(h_all=h_all, c_all=c_all)
+    return out
+
+
+def grid_rnn(x, ys, W, U, b, precision="f64", want_all=False):
+    """Grid RNN oracle (readings R12–R14).  x [B][Lx][H], ys [B][Ly][H], W [D][2][4][H][H],
+    U [D][2][4][2H][H], b [D][2][4][H]."""
+    dt = _prec(precision)
+    B, Lx, H = x.shape
+    Ly = ys.shape[1]
+    D = W.shape[0]
+    x, ys, W, U, b = (_c(a, dt) for a in (x, ys, W, U, b))
+    out = np.empty((B, Lx, Ly, 2, H), dt)
+    h_n = np.empty((B, D, 2, H), dt)
+    c_n = np.empty((B, D, 2, H), dt)
+    h_all = np.empty((B, D, Lx, Ly, 2, H), dt) if want_all else None
+    c_all = np.empty((B, D, Lx, Ly, 2, H), dt) if want_all else None
+    rc = getattr(lib(), f"ft_oracle_grid_rnn_{precision}")(
+        B, Lx, Ly, H, D, _p(x), _p(ys), _p(W), _p(U), _p(b), _p(out), _p(h_n), _p(c_n),
+        _p(h_all), _p(c_all))
+    if rc:
+        raise RuntimeError(f"oracle grid_rnn failed: {rc}")
+    res = dict(out=out, h_n=h_n, c_n=c_n)
+    if want_all:
+        res.update(h_all=h_all, c_all=c_all)
+    return res
+
+
+def lstm_cell(a, W4, hp, U4, b4, cp, precision="f64"):
+    """One cell (Listing 2).  a [Ka], W4 [4][Ka][H], hp [Kh] or None, U4 [4][Kh][H],
+    b4 [4][H], cp [H] or None.  Returns (h, c)."""
+    dt = _prec(precision)
+    H = b4.shape[1]
+    a = _c(a, dt)
+    W4 = _c(W4, dt)
+    U4 = _c(U4, dt)
+    b4 = _c(b4, dt)
+    hp = None if hp is None else _c(hp, dt)
+    cp = None if cp is None else _c(cp, dt)
+    h = np.empty(H, dt)
+    c = np.empty(H, dt)
+    z = np.empty(4 * H, dt)
+    Kh = U4.shape[1]
+    getattr(lib(), f"ft_oracle_lstm_cell_{precision}")(
+        H, _p(a), a.shape[0], _p(W4), _p(hp), Kh, _p(U4), _p(b4), _p(cp), _p(h), _p(c), _p(z))
+    return h, c

@@ -1,0 +1,346 @@
+"""Pins of the CPU oracle against things other than itself (SURVEY.md §8(c) c.6, P1–P11).
+
+Each test names the pin and the PAPER.md passage it checks.  Chosen so that a plausible
+mistake anywhere in the oracle (a dropped term, a swapped gate, a wrong time offset, a
+transposed weight, a missing bias, a wrong boundary state) fails at least one of them.
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import ftgen
+import oracle
+
+GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+
+
+def _sig(z):
+    return 1.0 / (1.0 + math.exp(-z))
+
+
+def _inputs(B=3, T=5, H=8, D=3, seed=7, scale=1.0, dtype="f32"):
+    return ftgen.stacked_inputs(B, T, H, D, seed, dtype=dtype, scale=scale)
+
+
+# --------------------------------------------------------------------------- P1
+def test_p1_zero_weights_zero_bias_gives_zero_state():
+    """P1 (closed form): W = U = 0, b = 0 ⇒ σ(0) = 1/2, tanh 0 = 0 ⇒ c ≡ 0, h ≡ 0
+    (Listing 2 L613–L615 with s0 = (0,0), L605)."""
+    p = _inputs()
+    for k in ("W", "U", "b"):
+        p[k] = np.zeros_like(p[k])
+    r = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    for k in ("y", "h_n", "c_n", "h_all", "c_all"):
+        assert np.all(r[k] == 0.0), k
+
+
+# --------------------------------------------------------------------------- P2
+@pytest.mark.parametrize("bias", [(0.3, 0.7, -0.2, 0.9), (-1.1, 2.0, 0.5, -0.6)])
+def test_p2_constant_gates_geometric_series(bias):
+    """P2 (closed form): W = U = 0, constant per-gate bias ⇒ constant gates i, f, o, ĝ;
+    c_t = i·ĝ·(1 − f^{t+1})/(1 − f), h_t = o·tanh(c_t), the same in every layer and row.
+    Pins the recurrence order, c_{-1} = 0 (L605) and the c/h formulas (L613–L615),
+    including the gate order (i, f, o, ĝ) = gs[0..3] (reading R1)."""
+    B, T, H, D = 2, 9, 4, 3
+    p = _inputs(B, T, H, D)
+    p["W"][:] = 0
+    p["U"][:] = 0
+    for g in range(4):
+        p["b"][:, g, :] = bias[g]
+    r = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    bi, bf, bo, bg = (float(np.float32(v)) for v in bias)
+    i, f, o, gh = _sig(bi), _sig(bf), _sig(bo), math.tanh(bg)
+    for t in range(T):
+        c_t = i * gh * (1 - f ** (t + 1)) / (1 - f)
+        h_t = o * math.tanh(c_t)
+        np.testing.assert_allclose(r["c_all"][:, :, t, :], c_t, rtol=0, atol=2e-15)
+        np.testing.assert_allclose(r["h_all"][:, :, t, :], h_t, rtol=0, atol=2e-15)
+
+
+# --------------------------------------------------------------------------- P3
+def _torch_lstm(p):
+    """torch.nn.LSTM in fp64 with the gate permutation (i,f,o,ĝ) → torch's (i,f,ĝ,o) (R1),
+    weight_ih = W[d][g]ᵀ (row-vector x@W convention, R5), bias_ih = b, bias_hh = 0 (R4)."""
+    import torch
+    x, W, U, b = (np.asarray(p[k], np.float64) for k in ("x", "W", "U", "b"))
+    B, T, H = x.shape
+    D = W.shape[0]
+    perm = (0, 1, 3, 2)
+    m = torch.nn.LSTM(H, H, num_layers=D, batch_first=True, dtype=torch.float64)
+    with torch.no_grad():
+        for d in range(D):
+            getattr(m, f"weight_ih_l{d}").copy_(torch.from_numpy(np.concatenate([W[d, g].T for g in perm])))
+            getattr(m, f"weight_hh_l{d}").copy_(torch.from_numpy(np.concatenate([U[d, g].T for g in perm])))
+            getattr(m, f"bias_ih_l{d}").copy_(torch.from_numpy(np.concatenate([b[d, g] for g in perm])))
+            getattr(m, f"bias_hh_l{d}").zero_()
+        y, (h_n, c_n) = m(torch.from_numpy(x))
+    return y.numpy(), h_n.permute(1, 0, 2).numpy(), c_n.permute(1, 0, 2).numpy()
+
+
+@pytest.mark.parametrize("shape", [(3, 7, 16, 3), (2, 5, 32, 2), (1, 1, 8, 1), (4, 3, 24, 5)])
+def test_p3_matches_torch_lstm_fp64(shape):
+    """P3 (library routine): the whole stacked LSTM — gates, wiring across depth (R6), outputs
+    (R8) — equals torch.nn.LSTM(num_layers=D) in fp64 (test-only cross-check)."""
+    B, T, H, D = shape
+    p = _inputs(B, T, H, D, seed=11, scale=2.0)
+    r = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"])
+    y, h_n, c_n = _torch_lstm(p)
+    np.testing.assert_allclose(r["y"], y, rtol=0, atol=1e-13)
+    np.testing.assert_allclose(r["h_n"], h_n, rtol=0, atol=1e-13)
+    np.testing.assert_allclose(r["c_n"], c_n, rtol=0, atol=1e-13)
+
+
+# --------------------------------------------------------------------------- P4
+def test_p4_forget_off_no_recurrence_is_batched_matmul():
+    """P4 (special case → batched matmul): U = 0 and b_f = −40 (f ≈ 4e-18) ⇒ for a one-layer
+    net h_t = o·tanh(i·ĝ) with gates from x@W + b (Listing 2: the input half of the GEMM
+    and the epilogue in isolation)."""
+    B, T, H = 3, 6, 16
+    p = _inputs(B, T, H, 1, seed=5, scale=2.0)
+    p["U"][:] = 0
+    p["b"][0, 1, :] = -40.0
+    r = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"])
+    x = p["x"].astype(np.float64)
+    z = np.einsum("btk,gkn->btgn", x, p["W"][0].astype(np.float64)) + p["b"][0].astype(np.float64)
+    sig = lambda v: 1 / (1 + np.exp(-v))
+    i, o, g = sig(z[:, :, 0]), sig(z[:, :, 2]), np.tanh(z[:, :, 3])
+    h = o * np.tanh(i * g)
+    np.testing.assert_allclose(r["y"], h, rtol=0, atol=1e-14)
+
+
+# --------------------------------------------------------------------------- P5
+def _run_schedule(p, order, dil=None):
+    """Re-run the nest cell by cell (oracle.lstm_cell) in a given legal order."""
+    x, W, U, b = (np.asarray(p[k], np.float64) for k in ("x", "W", "U", "b"))
+    B, T, H = x.shape
+    D = W.shape[0]
+    dil = dil or [1] * D
+    h = np.full((B, D, T, H), np.nan)
+    c = np.full((B, D, T, H), np.nan)
+    for bb in range(B):
+        for (d, t) in order(D, T):
+            s = dil[d]
+            a = x[bb, t] if d == 0 else h[bb, d - 1, t]
+            assert not np.any(np.isnan(a)), "schedule read an unwritten input"
+            hp = h[bb, d, t - s] if t >= s else None
+            cp = c[bb, d, t - s] if t >= s else None
+            if hp is not None:
+                assert not np.any(np.isnan(hp)), "schedule read an unwritten state"
+            h[bb, d, t], c[bb, d, t] = oracle.lstm_cell(a, W[d], hp, U[d], b[d], cp)
+    return h, c
+
+
+def _order_dt(D, T):
+    return [(d, t) for d in range(D) for t in range(T)]
+
+
+def _order_td(D, T):
+    return [(d, t) for t in range(T) for d in range(D)]
+
+
+def _order_wavefront(D, T):
+    """Hyperplane π(d,t) = d + t (T's first row [0,1,1,0], L341/L349), diagonals ascending."""
+    return [(d, k - d) for k in range(D + T - 1) for d in range(max(0, k - T + 1), min(k, D - 1) + 1)]
+
+
+@pytest.mark.parametrize("order", [_order_dt, _order_td, _order_wavefront])
+def test_p5_schedule_order_invariance(order):
+    """P5 (invariant): the nest is fully permutable (L333–L335), so executing the cells in
+    (d,t), (t,d) or wavefront order gives bitwise-identical results."""
+    p = _inputs(2, 6, 8, 4, seed=3, scale=2.0)
+    ref = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    h, c = _run_schedule(p, order)
+    assert np.array_equal(h, ref["h_all"])
+    assert np.array_equal(c, ref["c_all"])
+
+
+# --------------------------------------------------------------------------- P6
+def test_p6_batch_map_independence():
+    """P6 (invariant of `map`, Table 1): permuting batch rows permutes outputs
+    exactly; a row subset run alone equals those rows of the full run (bitwise).  This is what
+    makes full-size parity on sampled rows and batch sharding exact."""
+    p = _inputs(6, 5, 8, 3, seed=9)
+    full = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"])
+    perm = np.array([4, 0, 5, 2, 1, 3])
+    pr = oracle.stacked_lstm(p["x"][perm], p["W"], p["U"], p["b"])
+    for k in ("y", "h_n", "c_n"):
+        assert np.array_equal(pr[k], full[k][perm])
+    sub = [1, 4]
+    sr = oracle.stacked_lstm(p["x"][sub], p["W"], p["U"], p["b"])
+    for k in ("y", "h_n", "c_n"):
+        assert np.array_equal(sr[k], full[k][sub])
+
+
+# --------------------------------------------------------------------------- P7
+def test_p7a_dilation_one_equals_stacked():
+    """P7(a): all dilations 1 ⇒ the dilated nest (L331 with stride 1) is the stacked LSTM,
+    computed by an independent loop nest — bitwise equal."""
+    p = _inputs(3, 7, 8, 3, seed=2, scale=2.0)
+    a = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    b = oracle.dilated_rnn(p["x"], p["W"], p["U"], p["b"], [1, 1, 1], want_all=True)
+    for k in a:
+        assert np.array_equal(a[k], b[k]), k
+
+
+@pytest.mark.parametrize("s", [2, 3, 5])
+def test_p7b_single_layer_dilation_is_interleaved_lstms(s):
+    """P7(b): a one-layer LSTM with dilation s (strided access: dependence distance = stride,
+    L331) is s independent plain LSTMs over the subsequences x[:, r::s]."""
+    B, T, H = 2, 11, 8
+    p = _inputs(B, T, H, 1, seed=4, scale=2.0)
+    dl = oracle.dilated_rnn(p["x"], p["W"], p["U"], p["b"], [s])
+    for r in range(s):
+        sub = oracle.stacked_lstm(p["x"][:, r::s], p["W"], p["U"], p["b"])
+        assert np.array_equal(dl["y"][:, r::s], sub["y"])
+
+
+def test_p7c_dilation_at_least_T_has_no_recurrence():
+    """P7(c): T ≤ s_l ⇒ layer l never reads a recurrent state (t − s < 0 for every t, so the
+    zero initial state (h, c) = (0, 0) of R7 applies at every step): every time step is an
+    independent one-step (T = 1) network."""
+    p = _inputs(2, 4, 8, 2, seed=6, scale=2.0)
+    a = oracle.dilated_rnn(p["x"], p["W"], p["U"], p["b"], [4, 9])
+    for t in range(4):
+        b = oracle.stacked_lstm(p["x"][:, t:t + 1], p["W"], p["U"], p["b"])
+        assert np.array_equal(a["y"][:, t], b["y"][:, 0])
+    # and the recurrence matters once s < T
+    c = oracle.dilated_rnn(p["x"], p["W"], p["U"], p["b"], [1, 2])
+    assert not np.array_equal(a["y"], c["y"])
+
+
+def test_p7d_dilated_each_layer_matches_torch_on_subsequences():
+    """P7(d): a 2-layer dilated net, layer dilations (1, 2): layer 0 equals torch LSTM layer,
+    and layer 1 on the even/odd subsequences of layer-0's output equals a torch one-layer
+    LSTM — ties the strided access to an external library routine."""
+    B, T, H = 2, 8, 8
+    p = _inputs(B, T, H, 2, seed=8, scale=2.0)
+    r = oracle.dilated_rnn(p["x"], p["W"], p["U"], p["b"], [1, 2], want_all=True)
+    l0 = dict(x=p["x"], W=p["W"][:1], U=p["U"][:1], b=p["b"][:1])
+    y0, _, _ = _torch_lstm(l0)
+    np.testing.assert_allclose(r["h_all"][:, 0], y0, rtol=0, atol=1e-13)
+    for par in range(2):
+        l1 = dict(x=r["h_all"][:, 0, par::2], W=p["W"][1:], U=p["U"][1:], b=p["b"][1:])
+        y1, _, _ = _torch_lstm(l1)
+        np.testing.assert_allclose(r["h_all"][:, 1, par::2], y1, rtol=0, atol=1e-13)
+
+
+# --------------------------------------------------------------------------- P8
+def test_p8_grid_one_axis_reduces_to_stacked():
+    """P8 (reduction): grid with Ly = 1 ⇒ the h^x chain is a stacked LSTM over x with
+    U_d = U[d][x][rows 0:H] (the h^y part of s is the zero state); Lx = 1 ⇒ the h^y chain is a
+    stacked LSTM over ys with U_d = U[d][y][rows H:2H].  Bitwise (readings R12–R14)."""
+    B, L, H, D = 2, 6, 8, 3
+    g = ftgen.grid_inputs(B, L, 1, H, D, seed=12, dtype="f32", scale=2.0)
+    r = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"])
+    s = oracle.stacked_lstm(g["x"], g["W"][:, 0], g["U"][:, 0, :, :H, :], g["b"][:, 0])
+    assert np.array_equal(r["out"][:, :, 0, 0, :], s["y"])
+    assert np.array_equal(r["h_n"][:, :, 0, :], s["h_n"])
+    assert np.array_equal(r["c_n"][:, :, 0, :], s["c_n"])
+
+    g = ftgen.grid_inputs(B, 1, L, H, D, seed=13, dtype="f32", scale=2.0)
+    r = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"])
+    s = oracle.stacked_lstm(g["ys"], g["W"][:, 1], g["U"][:, 1, :, H:, :], g["b"][:, 1])
+    assert np.array_equal(r["out"][:, 0, :, 1, :], s["y"])
+    assert np.array_equal(r["h_n"][:, :, 1, :], s["h_n"])
+
+
+def test_p8b_grid_symmetry_swap_axes():
+    """P8(b) (invariant): swapping the roles of the two sequence axes (x↔ys, W/U/b axis 0↔1,
+    the two H-halves of s) transposes the grid: out'[j][i] = out[i][j] with axes swapped."""
+    B, Lx, Ly, H, D = 2, 3, 4, 8, 2
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, seed=14, dtype="f32", scale=2.0)
+    r = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"])
+    U2 = g["U"][:, ::-1].copy()
+    U2 = np.concatenate([U2[:, :, :, H:, :], U2[:, :, :, :H, :]], axis=3)
+    r2 = oracle.grid_rnn(g["ys"], g["x"], g["W"][:, ::-1], U2, g["b"][:, ::-1])
+    np.testing.assert_allclose(r2["out"], r["out"].transpose(0, 2, 1, 3, 4)[:, :, :, ::-1, :],
+                               rtol=0, atol=1e-14)
+
+
+# --------------------------------------------------------------------------- P9
+@pytest.mark.parametrize("beta", [0.4, -1.3])
+def test_p9_saturated_gates(beta):
+    """P9 (closed form): b_i = b_o = +40, b_f = −40, W = U = 0, b_ĝ = β ⇒ i = o = 1, f = 0
+    (to 4e-18) ⇒ c_t = tanh β, h_t = tanh(tanh β) at every t and depth (saturation paths)."""
+    p = _inputs(2, 5, 8, 3)
+    p["W"][:] = 0
+    p["U"][:] = 0
+    p["b"][:, 0] = 40
+    p["b"][:, 1] = -40
+    p["b"][:, 2] = 40
+    p["b"][:, 3] = beta
+    r = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    bt = float(np.float32(beta))
+    np.testing.assert_allclose(r["c_all"], math.tanh(bt), rtol=0, atol=1e-15)
+    np.testing.assert_allclose(r["h_all"], math.tanh(math.tanh(bt)), rtol=0, atol=1e-15)
+
+
+# --------------------------------------------------------------------------- P10
+def _table5_region3(L, D):
+    """Table 5 (L351–L358) transformed iteration space of region_3:
+    j4 ∈ [2, L+D−1), j3 ∈ [max(1, j4−L+1), min(j4, D)); depth = j3, time = j4 − j3."""
+    out = []
+    for j4 in range(2, L + D - 1):
+        for j3 in range(max(1, j4 - L + 1), min(j4, D)):
+            out.append((j3, j4 - j3))
+    return out
+
+
+def test_p10_table5_golden_enumeration():
+    """P10 (golden, tests/golden/table5_region3_L4_D3.txt, hand-enumerated from Table 5)."""
+    rows = []
+    with open(os.path.join(GOLDEN, "table5_region3_L4_D3.txt")) as f:
+        for line in f:
+            line = line.split("#")[0].strip()
+            if line:
+                rows.append(tuple(int(v) for v in line.split()))
+    got = [(j4, d, t) for (d, t) in _table5_region3(4, 3) for j4 in [d + t]]
+    assert got == rows
+
+
+@pytest.mark.parametrize("L,D", [(4, 3), (8, 2), (1, 5), (5, 1), (100, 16), (64, 8)])
+def test_p10_table5_covers_region3_once(L, D):
+    """P10 (brute force): Table 5's bounds enumerate region_3 = [1,D)×[1,L) (Fig. 4 range
+    constraints, L249–L254) exactly once; π = d + t orders every dependence (π·dep ≥ 1 for
+    dep ∈ {e_depth, e_time}, Table 4); the full grid has L+D−1 diagonals."""
+    cells = _table5_region3(L, D)
+    assert len(cells) == len(set(cells))
+    assert set(cells) == {(d, t) for d in range(1, D) for t in range(1, L)}
+    full = _order_wavefront(D, L)
+    assert len(full) == D * L and len(set(full)) == D * L
+    assert len({d + t for d, t in full}) == L + D - 1
+    for dep in [(1, 0), (0, 1)]:
+        assert dep[0] + dep[1] >= 1
+
+
+# --------------------------------------------------------------------------- P11
+def test_p11_fp32_headroom_for_1e4_tolerance():
+    """P11 (error analysis): the fp32 instantiation of the same nest (accurate expf/tanhf)
+    stays ≤ 1e-5 from fp64 on C1 — so the 1e-4 fp32 tolerance (BASELINE north_star) is
+    meetable by an fp32 kernel with accurate activations."""
+    c = ftgen.CONFIGS["C1"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C1"), "f32")
+    r64 = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="f64")
+    r32 = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="f32")
+    for k in r64:
+        assert np.max(np.abs(r64[k] - r32[k])) <= 1e-5, k
+
+
+def test_generator_is_counter_based_and_bf16_exact():
+    """The shared generator: element i depends only on (seed, stream, i); bf16 rounding is
+    RNE and idempotent; value ranges as DESIGN.md's input recipe states."""
+    a = ftgen.uniform(1, 2, 100)
+    b = ftgen.uniform(1, 2, 50, offset=50)
+    assert np.array_equal(a[50:], b)
+    assert np.all(a >= -1) and np.all(a < 1)
+    r = ftgen.round_bf16(a)
+    assert np.array_equal(ftgen.round_bf16(r), r)
+    assert np.max(np.abs(r - a)) <= 2.0 ** -8
+    # RNE tie: 1 + 2^-8 is halfway between 1 and 1 + 2^-7 -> rounds to even (1.0)
+    assert ftgen.round_bf16(np.array([1.0 + 2.0 ** -8]))[0] == 1.0
+    assert ftgen.round_bf16(np.array([1.0 + 3 * 2.0 ** -8]))[0] == 1.0 + 2.0 ** -6
+    p = ftgen.stacked_inputs(2, 3, 64, 2, 5, "bf16")
+    assert np.max(np.abs(p["W"])) <= 1 / 8 and np.max(np.abs(p["x"])) <= 1
+    ftgen.bf16_bits(p["W"])
