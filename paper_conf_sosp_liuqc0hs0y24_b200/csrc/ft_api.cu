@@ -1,0 +1,305 @@
+// ft_api.cu — the C ABI (include/ft.h): argument validation, workspace planning, problem
+// construction and kernel dispatch.  No compute happens here; every step of the path runs in
+// the kernels of wavefront_f32.cu / wavefront_bf16.cu.
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstring>
+#include <string>
+
+#include "../../include/ft.h"
+#include "ft_internal.h"
+
+#define FT_API extern "C" __attribute__((visibility("default")))
+
+namespace {
+
+thread_local std::string g_last_error = "no error";
+
+ft_status fail(ft_status s, const std::string& msg) {
+    g_last_error = msg;
+    return s;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+size_t round_up(size_t v, size_t a) { return (v + a - 1) / a * a; }
+
+size_t elem_size(ft_dtype dt) { return dt == FT_BF16 ? 2 : 4; }
+
+// Build the launch problem; returns OK or INVALID/UNSUPPORTED with g_last_error set.
+ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int* dil,
+                       ft_dtype dt, ft::Problem* p) {
+    if (dt != FT_F32 && dt != FT_BF16) return fail(FT_ERR_INVALID_ARGUMENT, "unknown dtype");
+    if (B <= 0 || L0 <= 0 || L1 <= 0 || H <= 0 || D <= 0)
+        return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    if (D > FT_MAX_DEPTH) return fail(FT_ERR_UNSUPPORTED, "depth > FT_MAX_DEPTH");
+    if (kind == ft::KIND_SEQ) {
+        if (!dil) return fail(FT_ERR_INVALID_ARGUMENT, "dilations is NULL");
+        for (int d = 0; d < D; ++d)
+            if (dil[d] < 1) return fail(FT_ERR_INVALID_ARGUMENT, "dilation < 1");
+    }
+    if (dt == FT_BF16 && H % 64 != 0)
+        return fail(FT_ERR_UNSUPPORTED, "bf16 path requires hidden % 64 == 0");
+    // 32-bit coordinate / index guards (TMA coordinates and row indices are int32)
+    const long long rows = (kind == ft::KIND_SEQ) ? (long long)D * L0 : (long long)D * L0 * L1 * 2;
+    if (rows > (1ll << 30) || (long long)B > (1ll << 30) || (long long)H > (1 << 20))
+        return fail(FT_ERR_UNSUPPORTED, "problem too large for 32-bit coordinates");
+
+    std::memset(p, 0, sizeof(*p));
+    p->kind = kind;
+    p->B = B;
+    p->H = H;
+    p->D = D;
+    p->L0 = L0;
+    p->L1 = L1;
+    p->naxes = (kind == ft::KIND_SEQ) ? 1 : 2;
+    p->BM = dt == FT_BF16 ? ft::BF16_BM : ft::F32_BM;
+    p->BNU = dt == FT_BF16 ? ft::BF16_BNU : ft::F32_BNU;
+    p->MB = (B + p->BM - 1) / p->BM;
+    p->NT = (H + p->BNU - 1) / p->BNU;
+    p->ncells = (long long)D * L0 * L1;
+    p->ntiles = p->ncells * p->naxes * p->MB * p->NT;
+    if (kind == ft::KIND_SEQ) {
+        int off = 0;
+        for (int d = 0; d < D; ++d) {
+            p->dil[d] = dil[d];
+            p->ring_off[d] = off;
+            const long long len = 2ll * dil[d] < L0 ? 2ll * dil[d] : L0;
+            off += (int)len;
+        }
+        p->ring_off[D] = off;
+    }
+    return FT_OK;
+}
+
+struct WsPlan {
+    size_t flags_off, flags_bytes;
+    size_t ring_off, ring_bytes;
+    size_t hall_off, hall_bytes;
+    size_t total;
+};
+
+WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
+    WsPlan w{};
+    w.flags_off = 0;
+    w.flags_bytes = round_up((size_t)p.ncells * p.MB * sizeof(int), 256);
+    w.ring_off = w.flags_off + w.flags_bytes;
+    w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
+    w.hall_off = w.ring_off + w.ring_bytes;
+    w.hall_bytes = h_all_provided
+                       ? 0
+                       : round_up((size_t)p.B * ft::h_rows(p) * p.H * elem_size(dt), 256);
+    w.total = w.hall_off + w.hall_bytes;
+    return w;
+}
+
+ft_status check_device() {
+    int dev = 0, major = 0, minor = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("no usable CUDA device: ") + cudaGetErrorString(e));
+    if (major != 10 || minor != 0)
+        return fail(FT_ERR_UNSUPPORTED, "this library is built for sm_100a (B200) only; device is sm_" +
+                                            std::to_string(major) + std::to_string(minor));
+    return FT_OK;
+}
+
+ft_status run(const ft::Problem& p, ft_dtype dt, ft::Tensors t, void* workspace,
+              size_t workspace_bytes, void* stream) {
+    const WsPlan w = plan_workspace(p, dt, t.h_all != nullptr);
+    if (w.total > 0 && !workspace) return fail(FT_ERR_INVALID_ARGUMENT, "workspace is NULL");
+    if (workspace && !aligned16(workspace))
+        return fail(FT_ERR_INVALID_ARGUMENT, "workspace not 16-byte aligned");
+    if (workspace_bytes < w.total)
+        return fail(FT_ERR_WORKSPACE_TOO_SMALL,
+                    "workspace_bytes " + std::to_string(workspace_bytes) + " < required " +
+                        std::to_string(w.total));
+    ft_status st = check_device();
+    if (st != FT_OK) return st;
+    uint8_t* ws = static_cast<uint8_t*>(workspace);
+    t.flags = reinterpret_cast<int*>(ws + w.flags_off);
+    t.c_ring = reinterpret_cast<float*>(ws + w.ring_off);
+    if (!t.h_all) t.h_all = ws + w.hall_off;
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    cudaError_t e = cudaMemsetAsync(t.flags, 0, w.flags_bytes, s);  // BK0: reset readiness flags
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("flag reset: ") + cudaGetErrorString(e));
+    std::string err;
+    e = (dt == FT_BF16) ? ft::launch_wavefront_bf16(p, t, s, &err)
+                        : ft::launch_wavefront_f32(p, t, s, &err);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, err.empty() ? cudaGetErrorString(e) : err);
+    return FT_OK;
+}
+
+#define REQUIRE_PTR(ptr, name)                                                               \
+    do {                                                                                     \
+        if (!(ptr)) return fail(FT_ERR_INVALID_ARGUMENT, std::string(name) + " is NULL");    \
+        if (!aligned16(ptr))                                                                 \
+            return fail(FT_ERR_INVALID_ARGUMENT, std::string(name) + " not 16-byte aligned"); \
+    } while (0)
+#define OPTIONAL_PTR(ptr, name)                                                              \
+    do {                                                                                     \
+        if ((ptr) && !aligned16(ptr))                                                        \
+            return fail(FT_ERR_INVALID_ARGUMENT, std::string(name) + " not 16-byte aligned"); \
+    } while (0)
+
+ft_status seq_fwd(int batch, int seq, int hidden, int depth, const int* dil, ft_dtype dt,
+                  const void* x, const void* W, const void* U, const float* b, void* y,
+                  void* h_n, float* c_n, void* h_all, float* c_all, void* workspace,
+                  size_t workspace_bytes, void* stream) {
+    ft::Problem p;
+    ft_status st = make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, dil, dt, &p);
+    if (st != FT_OK) return st;
+    REQUIRE_PTR(x, "x");
+    REQUIRE_PTR(W, "W");
+    REQUIRE_PTR(U, "U");
+    REQUIRE_PTR(b, "b");
+    REQUIRE_PTR(y, "y");
+    REQUIRE_PTR(h_n, "h_n");
+    REQUIRE_PTR(c_n, "c_n");
+    OPTIONAL_PTR(h_all, "h_all");
+    OPTIONAL_PTR(c_all, "c_all");
+    ft::Tensors t;
+    t.x = x;
+    t.W = W;
+    t.U = U;
+    t.b = b;
+    t.y = y;
+    t.h_n = h_n;
+    t.c_n = c_n;
+    t.h_all = h_all;
+    t.c_all = c_all;
+    return run(p, dt, t, workspace, workspace_bytes, stream);
+}
+
+}  // namespace
+
+namespace ft {
+long long c_ring_elems(const Problem& p) {
+    if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * p.B * p.H;
+    return (long long)p.D * 2 * p.L1 * p.B * p.H + (long long)p.D * p.L0 * 2 * p.B * p.H;
+}
+}  // namespace ft
+
+FT_API int ft_version(void) { return FT_VERSION; }
+
+FT_API const char* ft_status_string(ft_status s) {
+    switch (s) {
+        case FT_OK: return "FT_OK";
+        case FT_ERR_INVALID_ARGUMENT: return "FT_ERR_INVALID_ARGUMENT";
+        case FT_ERR_UNSUPPORTED: return "FT_ERR_UNSUPPORTED";
+        case FT_ERR_CUDA: return "FT_ERR_CUDA";
+        case FT_ERR_WORKSPACE_TOO_SMALL: return "FT_ERR_WORKSPACE_TOO_SMALL";
+    }
+    return "FT_ERR_UNKNOWN";
+}
+
+FT_API const char* ft_last_error(void) { return g_last_error.c_str(); }
+
+FT_API size_t ft_stacked_lstm_workspace_size(int batch, int seq, int hidden, int depth, ft_dtype dt,
+                                             int h_all_provided) {
+    if (depth <= 0 || depth > FT_MAX_DEPTH) return 0;
+    int ones[FT_MAX_DEPTH];
+    for (int d = 0; d < depth; ++d) ones[d] = 1;
+    ft::Problem p;
+    if (make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, ones, dt, &p) != FT_OK) return 0;
+    return plan_workspace(p, dt, h_all_provided != 0).total;
+}
+
+FT_API ft_status ft_stacked_lstm_fwd(int batch, int seq, int hidden, int depth, ft_dtype dt,
+                                     const void* x, const void* W, const void* U, const float* b,
+                                     void* y, void* h_n, float* c_n, void* h_all, float* c_all,
+                                     void* workspace, size_t workspace_bytes, void* stream) {
+    if (depth <= 0) return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    if (depth > FT_MAX_DEPTH) return fail(FT_ERR_UNSUPPORTED, "depth > FT_MAX_DEPTH");
+    int ones[FT_MAX_DEPTH];
+    for (int d = 0; d < depth; ++d) ones[d] = 1;
+    return seq_fwd(batch, seq, hidden, depth, ones, dt, x, W, U, b, y, h_n, c_n, h_all, c_all,
+                   workspace, workspace_bytes, stream);
+}
+
+FT_API size_t ft_dilated_rnn_workspace_size(int batch, int seq, int hidden, int depth,
+                                            const int* dilations, ft_dtype dt, int h_all_provided) {
+    ft::Problem p;
+    if (make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, dilations, dt, &p) != FT_OK) return 0;
+    return plan_workspace(p, dt, h_all_provided != 0).total;
+}
+
+FT_API ft_status ft_dilated_rnn_fwd(int batch, int seq, int hidden, int depth, const int* dilations,
+                                    ft_dtype dt, const void* x, const void* W, const void* U,
+                                    const float* b, void* y, void* h_n, float* c_n, void* h_all,
+                                    float* c_all, void* workspace, size_t workspace_bytes,
+                                    void* stream) {
+    return seq_fwd(batch, seq, hidden, depth, dilations, dt, x, W, U, b, y, h_n, c_n, h_all, c_all,
+                   workspace, workspace_bytes, stream);
+}
+
+FT_API size_t ft_grid_rnn_workspace_size(int batch, int len_x, int len_y, int hidden, int depth,
+                                         ft_dtype dt, int h_all_provided) {
+    ft::Problem p;
+    if (make_problem(ft::KIND_GRID, batch, len_x, len_y, hidden, depth, nullptr, dt, &p) != FT_OK)
+        return 0;
+    return plan_workspace(p, dt, h_all_provided != 0).total;
+}
+
+FT_API ft_status ft_grid_rnn_fwd(int batch, int len_x, int len_y, int hidden, int depth, ft_dtype dt,
+                                 const void* x, const void* ys, const void* W, const void* U,
+                                 const float* b, void* out, void* h_n, float* c_n, void* h_all,
+                                 float* c_all, void* workspace, size_t workspace_bytes,
+                                 void* stream) {
+    ft::Problem p;
+    ft_status st = make_problem(ft::KIND_GRID, batch, len_x, len_y, hidden, depth, nullptr, dt, &p);
+    if (st != FT_OK) return st;
+    REQUIRE_PTR(x, "x");
+    REQUIRE_PTR(ys, "ys");
+    REQUIRE_PTR(W, "W");
+    REQUIRE_PTR(U, "U");
+    REQUIRE_PTR(b, "b");
+    REQUIRE_PTR(out, "out");
+    REQUIRE_PTR(h_n, "h_n");
+    REQUIRE_PTR(c_n, "c_n");
+    OPTIONAL_PTR(h_all, "h_all");
+    OPTIONAL_PTR(c_all, "c_all");
+    ft::Tensors t;
+    t.x = x;
+    t.ys = ys;
+    t.W = W;
+    t.U = U;
+    t.b = b;
+    t.y = out;
+    t.h_n = h_n;
+    t.c_n = c_n;
+    t.h_all = h_all;
+    t.c_all = c_all;
+    return run(p, dt, t, workspace, workspace_bytes, stream);
+}
+
+FT_API long long ft_wavefront_cells(int kind, int depth, int len_a, int len_b, int* out_cells,
+                                    long long cap) {
+    if (kind != ft::KIND_SEQ && kind != ft::KIND_GRID) return -1;
+    if (kind == ft::KIND_SEQ) len_b = 1;
+    if (depth <= 0 || len_a <= 0 || len_b <= 0 || depth > FT_MAX_DEPTH) return -1;
+    if (cap > 0 && !out_cells) return -1;
+    ft::Problem p;
+    std::memset(&p, 0, sizeof(p));
+    p.kind = kind;
+    p.D = depth;
+    p.L0 = len_a;
+    p.L1 = len_b;
+    p.B = p.H = 1;
+    p.naxes = kind == ft::KIND_SEQ ? 1 : 2;
+    p.MB = p.NT = 1;
+    p.ncells = (long long)depth * len_a * len_b;
+    ft::Cursor cur = ft::cursor_begin();
+    for (long long o = 0; o < p.ncells; ++o) {
+        ft::cursor_seek(p, cur, o);
+        if (o < cap) {
+            out_cells[4 * o + 0] = cur.cell.k;
+            out_cells[4 * o + 1] = cur.cell.d;
+            out_cells[4 * o + 2] = cur.cell.i;
+            out_cells[4 * o + 3] = cur.cell.j;
+        }
+    }
+    return p.ncells;
+}

@@ -1,0 +1,307 @@
+// ft_common.cuh — problem description, wavefront cell order and readiness-flag protocol shared
+// by every kernel of the library (host + device).  Nothing here is shared with oracle/.
+//
+// The schedule is the paper's reordering result (§5.2): the nest
+// map(batch) ∘ scan(depth) ∘ scan(time) is fully permutable (L333–L335) with constant
+// dependence distances (Table 4), so one transformed dimension — the hyperplane
+// π = d + t (T's first row [0,1,1,0], L341/L349) — carries every dependence.  Cells are handed
+// out diagonal by diagonal; inside a diagonal every cell is independent (Fig. 9: "cells of
+// the same colour run in parallel").  The batch dimension, whose null-space carries the weight
+// reuse (L345–L349), is the GEMM M dimension inside a cell.
+#pragma once
+
+#include <cstdint>
+
+#include "../../include/ft.h"
+
+#ifdef __CUDACC__
+#define FT_HD __host__ __device__ __forceinline__
+#else
+#define FT_HD inline
+#endif
+
+namespace ft {
+
+enum Kind : int { KIND_SEQ = 0 /* stacked + dilated */, KIND_GRID = 1 };
+
+// One launch's problem.  All sizes in elements.
+struct Problem {
+    int kind;
+    int B, H, D;
+    int L0, L1;          // KIND_SEQ: L0 = seq, L1 = 1.  KIND_GRID: L0 = len_x, L1 = len_y.
+    int naxes;           // 1 (seq) or 2 (grid)
+    int BM, BNU;         // batch rows and hidden units per tile (kernel-specific)
+    int MB, NT;          // m-blocks = ceil(B/BM), n-tiles per axis = ceil(H/BNU)
+    long long ncells;    // D*L0*L1
+    long long ntiles;    // ncells * naxes * MB * NT
+    int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)
+    int ring_off[FT_MAX_DEPTH + 1];  // KIND_SEQ: c-ring slot offset per layer; ring_len = diff
+};
+
+struct Cell {
+    int k, d, i, j;   // diagonal, depth, position (i = t for KIND_SEQ; j = 0)
+};
+
+FT_HD int num_diagonals(const Problem& p) {
+    return p.kind == KIND_SEQ ? p.D + p.L0 - 1 : p.D + p.L0 + p.L1 - 2;
+}
+
+FT_HD int imax(int a, int b) { return a > b ? a : b; }
+FT_HD int imin(int a, int b) { return a < b ? a : b; }
+
+// First cell (k = 0): (0, 0, 0, 0).
+FT_HD Cell first_cell() { return Cell{0, 0, 0, 0}; }
+
+// Successor of `c` in wavefront order: diagonal ascending; within a diagonal depth ascending,
+// then i ascending.  For KIND_SEQ the cells of diagonal k are d ∈ [max(0, k-L+1), min(k, D-1)]
+// with t = k - d — exactly Table 5's bounds (L355–L358) extended to the boundary regions.
+FT_HD Cell next_cell(const Problem& p, Cell c) {
+    if (p.kind == KIND_SEQ) {
+        const int dhi = imin(c.k, p.D - 1);
+        if (c.d < dhi) {
+            c.d += 1;
+        } else {
+            c.k += 1;
+            c.d = imax(0, c.k - p.L0 + 1);
+        }
+        c.i = c.k - c.d;
+        c.j = 0;
+        return c;
+    }
+    // KIND_GRID: diagonal k = d + i + j.
+    const int r = c.k - c.d;
+    if (c.i < imin(r, p.L0 - 1)) {
+        c.i += 1;
+        c.j = r - c.i;
+        return c;
+    }
+    for (;;) {
+        if (c.d < imin(c.k, p.D - 1)) {
+            c.d += 1;
+        } else {
+            c.k += 1;
+            c.d = imax(0, c.k - (p.L0 - 1) - (p.L1 - 1));
+        }
+        const int rr = c.k - c.d;
+        const int ilo = imax(0, rr - (p.L1 - 1));
+        const int ihi = imin(rr, p.L0 - 1);
+        if (ilo <= ihi) {
+            c.i = ilo;
+            c.j = rr - ilo;
+            return c;
+        }
+    }
+}
+
+// Linear cell index used for flags: KIND_SEQ d*L0 + t, KIND_GRID (d*L0 + i)*L1 + j.
+FT_HD long long cell_lin(const Problem& p, int d, int i, int j) {
+    return ((long long)d * p.L0 + i) * p.L1 + j;
+}
+
+FT_HD int tiles_per_cell(const Problem& p) { return p.naxes * p.MB * p.NT; }
+
+// Flags: one int per (cell, m-block); complete when it reaches naxes * NT.
+FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT; }
+
+// Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).
+struct Cursor {
+    long long ord;  // ordinal of `cell` in wavefront order
+    Cell cell;
+};
+
+FT_HD Cursor cursor_begin() { return Cursor{0, first_cell()}; }
+
+FT_HD void cursor_seek(const Problem& p, Cursor& cur, long long target_ord) {
+    while (cur.ord < target_ord) {
+        cur.cell = next_cell(p, cur.cell);
+        ++cur.ord;
+    }
+}
+
+// Decomposition of the within-cell index w = (axis * MB + m) * NT + n.
+struct TileId {
+    Cell cell;
+    int axis, m, n;
+};
+
+FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
+    const int tpc = tiles_per_cell(p);
+    cursor_seek(p, cur, tile / tpc);
+    int w = (int)(tile % tpc);
+    TileId t;
+    t.cell = cur.cell;
+    t.n = w % p.NT;
+    w /= p.NT;
+    t.m = w % p.MB;
+    t.axis = w / p.MB;
+    return t;
+}
+
+// Producer cells of (d, i, j) — the dependence vectors of Table 4 (L307–L317):
+// KIND_SEQ: e_depth → (d-1, t), s_d·e_time → (d, t - s_d) (strided access, L331).
+// KIND_GRID: e_depth, e_x, e_y → (d-1,i,j), (d,i-1,j), (d,i,j-1).
+// Returns the number of producers written to out[] (as linear cell indices).
+FT_HD int producers(const Problem& p, const Cell& c, long long out[3]) {
+    int n = 0;
+    if (c.d > 0) out[n++] = cell_lin(p, c.d - 1, c.i, c.j);
+    if (p.kind == KIND_SEQ) {
+        const int s = p.dil[c.d];
+        if (c.i >= s) out[n++] = cell_lin(p, c.d, c.i - s, 0);
+    } else {
+        if (c.i > 0) out[n++] = cell_lin(p, c.d, c.i - 1, c.j);
+        if (c.j > 0) out[n++] = cell_lin(p, c.d, c.i, c.j - 1);
+    }
+    return n;
+}
+
+// ------------------------------------------------------------------------------------------
+// Access materialization (§5.3): the access maps of Fig. 4 (e12 o=[0,-1,0],
+// e13 o=[0,0,-1], e14 ws[d], e15 the SSA write, L249–L254) become row coordinates into the
+// batch-outermost buffers.  An activation "row" is the middle coordinate of the
+// (hidden, rows, batch) view of a buffer: x/ys: position; h_all: (d, t) or (d, i, j, axis).
+// ------------------------------------------------------------------------------------------
+enum Src : int { SRC_X = 0, SRC_YS = 1, SRC_H = 2 };
+enum WSel : int { W_IN = 0, W_REC = 1 };
+
+struct Segment {
+    int src;    // Src
+    int row;    // middle coordinate in the source's (H, rows, B) view
+    int wsel;   // WSel
+    int slice;  // weight slice: d (seq) or d*2+axis (grid)
+    int krow0;  // first K row inside the weight slice (grid U: 0 for h^x, H for h^y)
+};
+
+// rows per batch row of h_all
+FT_HD int h_rows(const Problem& p) {
+    return p.kind == KIND_SEQ ? p.D * p.L0 : p.D * p.L0 * p.L1 * 2;
+}
+FT_HD int h_row(const Problem& p, int d, int i, int j, int a) {
+    return p.kind == KIND_SEQ ? d * p.L0 + i : ((d * p.L0 + i) * p.L1 + j) * 2 + a;
+}
+// K rows of one U slice: H (seq) or 2H (grid, acting on s = [h^x; h^y]).
+FT_HD int u_krows(const Problem& p) { return p.kind == KIND_SEQ ? p.H : 2 * p.H; }
+
+// The A-operand segments of one tile (the vertical merge x@w + h@u of L609 as one K loop).
+// A segment whose producer is outside the domain (t < s, i = 0, j = 0) is the zero initial
+// state (scanl s0 = 0, L159/L605) and is skipped: that is the paper's boundary region split
+// (region_0..3, L243/L256).
+FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
+    const Cell& c = tl.cell;
+    int n = 0;
+    if (p.kind == KIND_SEQ) {
+        seg[n++] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0}
+                              : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0};
+        const int s = p.dil[c.d];
+        if (c.i >= s) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i - s, 0, 0), W_REC, c.d, 0};
+        return n;
+    }
+    const int a = tl.axis, sl = c.d * 2 + a;
+    if (c.d == 0)
+        seg[n++] = Segment{a == 0 ? SRC_X : SRC_YS, a == 0 ? c.i : c.j, W_IN, sl, 0};
+    else
+        seg[n++] = Segment{SRC_H, h_row(p, c.d - 1, c.i, c.j, a), W_IN, sl, 0};
+    if (c.i > 0) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i - 1, c.j, 0), W_REC, sl, 0};
+    if (c.j > 0) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i, c.j - 1, 1), W_REC, sl, p.H};
+    return n;
+}
+
+// rows per batch row of each activation source
+FT_HD int src_rows(const Problem& p, int src) {
+    return src == SRC_X ? p.L0 : (src == SRC_YS ? p.L1 : h_rows(p));
+}
+
+// Cell-state ring (fp32).  KIND_SEQ: layer d owns ring_len_d = min(T, 2·s_d) slots
+// [ring_off[d], ring_off[d+1]); slot of step t is t mod ring_len_d.  The slot written by
+// (d, t) last held c(d, t - 2s_d), read by (d, t - s_d) — a direct producer of (d, t), so the
+// reuse is ordered by the flag protocol.  KIND_GRID: c^x ring of 2 slots over i
+// ([D][2][Ly][B][H]) and c^y ring of 2 slots over j ([D][Lx][2][B][H]), same argument.
+FT_HD long long c_ring_index(const Problem& p, int d, int i, int j, int a, int b, int n) {
+    if (p.kind == KIND_SEQ) {
+        const int len = p.ring_off[d + 1] - p.ring_off[d];
+        const long long slot = p.ring_off[d] + i % len;
+        return (slot * p.B + b) * (long long)p.H + n;
+    }
+    if (a == 0)
+        return ((((long long)d * 2 + (i & 1)) * p.L1 + j) * p.B + b) * (long long)p.H + n;
+    const long long base = (long long)p.D * 2 * p.L1 * p.B * p.H;
+    return base + ((((long long)d * p.L0 + i) * 2 + (j & 1)) * p.B + b) * (long long)p.H + n;
+}
+
+// The cell whose c the tile's epilogue reads (its c-producer), or -1 (zero initial state).
+FT_HD long long c_producer(const Problem& p, const TileId& tl, int* pi, int* pj) {
+    const Cell& c = tl.cell;
+    if (p.kind == KIND_SEQ) {
+        const int s = p.dil[c.d];
+        if (c.i < s) return -1;
+        *pi = c.i - s;
+        *pj = 0;
+        return cell_lin(p, c.d, c.i - s, 0);
+    }
+    if (tl.axis == 0) {
+        if (c.i == 0) return -1;
+        *pi = c.i - 1;
+        *pj = c.j;
+        return cell_lin(p, c.d, c.i - 1, c.j);
+    }
+    if (c.j == 0) return -1;
+    *pi = c.i;
+    *pj = c.j - 1;
+    return cell_lin(p, c.d, c.i, c.j - 1);
+}
+
+// Output element indices (batch row b, unit n).
+FT_HD long long h_all_index(const Problem& p, const Cell& c, int a, int b, int n) {
+    return ((long long)b * h_rows(p) + h_row(p, c.d, c.i, c.j, a)) * p.H + n;
+}
+// y (seq, top layer) / out (grid, top depth); valid only when c.d == D-1.
+FT_HD long long y_index(const Problem& p, const Cell& c, int a, int b, int n) {
+    if (p.kind == KIND_SEQ) return ((long long)b * p.L0 + c.i) * p.H + n;
+    return ((((long long)b * p.L0 + c.i) * p.L1 + c.j) * 2 + a) * (long long)p.H + n;
+}
+// h_n / c_n; valid only at the last position.
+FT_HD bool is_last_pos(const Problem& p, const Cell& c) {
+    return p.kind == KIND_SEQ ? c.i == p.L0 - 1 : (c.i == p.L0 - 1 && c.j == p.L1 - 1);
+}
+FT_HD long long hn_index(const Problem& p, const Cell& c, int a, int b, int n) {
+    return ((long long)b * p.D + c.d) * (long long)p.naxes * p.H + (long long)a * p.H + n;
+}
+
+}  // namespace ft
+
+#ifdef __CUDACC__
+namespace ft {
+
+#ifndef FT_SPIN_TIMEOUT_NS
+#define FT_SPIN_TIMEOUT_NS 20000000000ull  // 20 s: a lost dependency traps instead of hanging
+#endif
+
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+__device__ __forceinline__ int ld_acquire_gpu(const int* p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void red_release_gpu_add(int* p, int v) {
+    asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Bounded acquire-spin on a readiness counter.
+__device__ __forceinline__ void wait_flag_geq(const int* p, int target) {
+    if (ld_acquire_gpu(p) >= target) return;
+    const uint64_t t0 = globaltimer_ns();
+    for (;;) {
+#pragma unroll 1
+        for (int it = 0; it < 256; ++it)
+            if (ld_acquire_gpu(p) >= target) return;
+        if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
+    }
+}
+
+}  // namespace ft
+#endif

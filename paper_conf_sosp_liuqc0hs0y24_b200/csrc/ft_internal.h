@@ -1,0 +1,40 @@
+// ft_internal.h — declarations shared by the library's translation units (not installed).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <string>
+
+#include "ft_common.cuh"
+
+namespace ft {
+
+// Device pointers of one call.  `y` is `out` for the grid call.
+struct Tensors {
+    const void* x = nullptr;
+    const void* ys = nullptr;
+    const void* W = nullptr;
+    const void* U = nullptr;
+    const float* b = nullptr;
+    void* y = nullptr;
+    void* h_n = nullptr;
+    float* c_n = nullptr;
+    void* h_all = nullptr;   // never NULL at launch (workspace stand-in if the caller passed NULL)
+    float* c_all = nullptr;  // optional
+    float* c_ring = nullptr; // workspace: fp32 cell-state ring
+    int* flags = nullptr;    // workspace: readiness counters [ncells][MB]
+};
+
+// Tile shapes of the two kernels.
+constexpr int F32_BM = 32, F32_BNU = 32;     // SIMT correctness path (BK1)
+constexpr int BF16_BM = 128, BF16_BNU = 64;  // tcgen05 path (BK2–BK4)
+
+// Number of fp32 ring elements the cell state needs.
+long long c_ring_elems(const Problem& p);
+
+cudaError_t launch_wavefront_f32(const Problem& p, const Tensors& t, cudaStream_t s,
+                                 std::string* err);
+cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
+                                  std::string* err);
+
+}  // namespace ft

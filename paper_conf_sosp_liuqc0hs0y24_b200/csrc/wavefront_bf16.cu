@@ -1,0 +1,413 @@
+// wavefront_bf16.cu — BK2/BK3/BK4: the persistent sm_100a wavefront (stacked, dilated, grid).
+//
+// One launch runs the whole nest.  Every CTA (one per SM, cooperative launch so all are
+// co-resident) walks the global tile sequence in wavefront order (ft_common.cuh) with stride
+// gridDim.x.  A tile = (cell, axis, 128 batch rows, 64 hidden units x 4 gates):
+//
+//   z[128 x 256] = Σ_seg A_seg[128 x H] · B_seg[H x 256] + b          (Listing 2)
+//
+// the horizontal merge of the 4 gate maps (N = 4 x 64, L287) and the vertical merge of
+// x@w + h@u (K = segments x H, L289–L293) as one tcgen05 GEMM; A = activation rows (batch =
+// the GEMM M dimension, the reuse dimension of L345–L349), B = the weight slice W[d][g][k][n]
+// used as an MN-major operand (n contiguous, no repacking).  The pointwise LSTM update
+// (L611–L615) runs in the epilogue straight out of TMEM.
+//
+// Warp roles (192 threads):
+//   warp 0      TMA producer: waits the tile's producer cells (readiness flags), then streams
+//               K-chunks of A (128 rows x 64 k, 16 KiB) and B (4 gates x 64 k x 64 n, 32 KiB)
+//               into a 4-stage shared-memory ring (mbarrier full/empty).
+//   warp 1      MMA issuer: one thread issues tcgen05.mma (M128 N256 K16) into a TMEM
+//               accumulator, double-buffered (2 x 256 columns) so tile n+1's MMAs overlap
+//               tile n's epilogue.
+//   warps 2-5   epilogue: tcgen05.ld → +b, σ/σ/σ/tanh, c' = f·c + i·ĝ, h' = o·tanh(c')
+//               (fp32 registers), h' → bf16 → h_all (the SSA buffer node, L217) and y / h_n;
+//               c' → fp32 cell-state ring (+ c_all / c_n); then release the tile's share of the
+//               (cell, m-block) readiness counter.
+//
+// Cross-CTA ordering (generic-proxy stores → another SM's async-proxy TMA loads):
+//   writer: st.global …; fence.acq_rel.gpu (every thread); bar.sync; red.release.gpu
+//   reader: ld.acquire.gpu (bounded spin); fence.proxy.async.global; cp.async.bulk.tensor
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <string>
+
+#include "ft_internal.h"
+#include "ft_sm100.cuh"
+
+namespace ft {
+namespace {
+
+using namespace sm100;
+
+constexpr int BM = BF16_BM;    // 128 batch rows = TMEM lanes = UMMA M
+constexpr int BNU = BF16_BNU;  // 64 hidden units per tile
+constexpr int BN = 4 * BNU;    // 256 = UMMA N (i | f | o | ĝ)
+constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16
+constexpr int UK = 16;         // UMMA K for kind::f16
+constexpr int STAGES = 4;
+constexpr int A_BYTES = BM * BK * 2;  // 16 KiB
+constexpr int B_BYTES = BN * BK * 2;  // 32 KiB
+constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+constexpr int THREADS = 192;
+constexpr int TMEM_COLS = 2 * BN;  // double-buffered accumulator
+constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024;
+constexpr uint32_t IDESC = make_idesc_bf16_f32(BM, BN, /*a MN-major*/ false, /*b MN-major*/ true);
+
+struct Maps {
+    CUtensorMap x, ys, h, W, U;
+};
+
+// ------------------------------------------------------------------------------ producer
+__device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
+                                             uint8_t* sA, uint8_t* sB, uint64_t* full,
+                                             uint64_t* empty) {
+    int stage = 0;
+    uint32_t phase = 0;
+    Cursor cur = cursor_begin();
+    const int target = flag_target(P);
+    const int kchunks = P.H / BK;
+    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+        const TileId tl = decode_tile(P, cur, tile);
+        long long prod[3];
+        const int np = producers(P, tl.cell, prod);
+        for (int q = 0; q < np; ++q) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
+        fence_proxy_async_global();
+        Segment seg[3];
+        const int ns = segments(P, tl, seg);
+        for (int s = 0; s < ns; ++s) {
+            const CUtensorMap* am = seg[s].src == SRC_X ? &M.x : (seg[s].src == SRC_YS ? &M.ys : &M.h);
+            const CUtensorMap* bm = seg[s].wsel == W_IN ? &M.W : &M.U;
+            for (int kc = 0; kc < kchunks; ++kc) {
+                mbar_wait(&empty[stage], phase ^ 1);
+                mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
+                tma_load_3d(sA + stage * A_BYTES, am, &full[stage], kc * BK, seg[s].row, tl.m * BM);
+                tma_load_4d(sB + stage * B_BYTES, bm, &full[stage], tl.n * BNU,
+                            seg[s].krow0 + kc * BK, 0, seg[s].slice);
+                if (++stage == STAGES) {
+                    stage = 0;
+                    phase ^= 1;
+                }
+            }
+        }
+    }
+}
+
+// ------------------------------------------------------------------------------ MMA issuer
+__device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, uint8_t* sA,
+                                        uint8_t* sB, uint64_t* full, uint64_t* empty,
+                                        uint64_t* tfull, uint64_t* tempty) {
+    int stage = 0;
+    uint32_t phase = 0;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    Cursor cur = cursor_begin();
+    const int kchunks = P.H / BK;
+    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+        const TileId tl = decode_tile(P, cur, tile);
+        Segment seg[3];
+        const int nchunks = segments(P, tl, seg) * kchunks;
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+        for (int c = 0; c < nchunks; ++c) {
+            mbar_wait(&full[stage], phase);
+            tc_fence_after();
+            // A: K-major, SW128: rows of 128 B, 8-row groups 1024 B apart (SBO); K step = +32 B.
+            // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups
+            //    1024 B apart (SBO); K step of 16 rows = +2048 B.
+            const uint64_t ad = make_sdesc(smem_u32(sA + stage * A_BYTES), 16, 1024);
+            const uint64_t bd = make_sdesc(smem_u32(sB + stage * B_BYTES), 8192, 1024);
+#pragma unroll
+            for (int kk = 0; kk < BK / UK; ++kk)
+                umma_f16(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
+                         bd + (uint64_t)((kk * UK * 128) >> 4), IDESC, (c | kk) != 0);
+            umma_commit(&empty[stage]);
+            if (++stage == STAGES) {
+                stage = 0;
+                phase ^= 1;
+            }
+        }
+        umma_commit(&tfull[acc]);
+        acc ^= 1;
+        if (acc == 0) acc_phase ^= 1;
+    }
+}
+
+// ------------------------------------------------------------------------------ epilogue
+__device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
+    __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);  // RNE
+    return *reinterpret_cast<uint32_t*>(&v);
+}
+
+__device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
+                                             uint64_t* tfull, uint64_t* tempty) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int q = warp & 3;  // TMEM lane quadrant this warp may access
+    const int row = q * 32 + lane;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    Cursor cur = cursor_begin();
+    const int target = flag_target(P);
+    __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
+    __nv_bfloat16* y = (__nv_bfloat16*)T.y;
+    __nv_bfloat16* h_n = (__nv_bfloat16*)T.h_n;
+    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+        const TileId tl = decode_tile(P, cur, tile);
+        const Cell c = tl.cell;
+        int ci = 0, cj = 0;
+        const long long cprod = c_producer(P, tl, &ci, &cj);
+        if (cprod >= 0) wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
+        mbar_wait(&tfull[acc], acc_phase);
+        tc_fence_after();
+
+        const int b = tl.m * BM + row;
+        const bool valid = b < P.B;
+        const int slice = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
+        const float* bias = T.b + (long long)slice * 4 * P.H;
+        const bool top = (c.d == P.D - 1), last = is_last_pos(P, c);
+        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16);
+#pragma unroll 1
+        for (int u0 = 0; u0 < BNU; u0 += 16) {
+            __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
+            float zi[16], zf[16], zo[16], zg[16];
+            tmem_ld_32x32b_x16(tbase + 0 * BNU + u0, zi);
+            tmem_ld_32x32b_x16(tbase + 1 * BNU + u0, zf);
+            tmem_ld_32x32b_x16(tbase + 2 * BNU + u0, zo);
+            tmem_ld_32x32b_x16(tbase + 3 * BNU + u0, zg);
+            tmem_wait_ld();
+            if (u0 + 16 == BNU) {  // accumulator buffer drained → hand it back to the MMA warp
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&tempty[acc]);
+            }
+            if (valid) {
+            const int n = tl.n * BNU + u0;
+            float cp[16];
+            if (cprod >= 0) {
+                const float4* src = reinterpret_cast<const float4*>(
+                    T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n));
+#pragma unroll
+                for (int v = 0; v < 4; ++v) {
+                    const float4 t4 = __ldcg(src + v);
+                    cp[4 * v + 0] = t4.x; cp[4 * v + 1] = t4.y;
+                    cp[4 * v + 2] = t4.z; cp[4 * v + 3] = t4.w;
+                }
+            } else {
+#pragma unroll
+                for (int v = 0; v < 16; ++v) cp[v] = 0.f;
+            }
+            float hv[16], cv[16];
+#pragma unroll
+            for (int v = 0; v < 16; ++v) {
+                const float ig = sigmoid_approx(zi[v] + __ldg(bias + 0 * P.H + n + v));
+                const float fg = sigmoid_approx(zf[v] + __ldg(bias + 1 * P.H + n + v));
+                const float og = sigmoid_approx(zo[v] + __ldg(bias + 2 * P.H + n + v));
+                const float gh = tanh_approx(zg[v] + __ldg(bias + 3 * P.H + n + v));
+                const float cn = fmaf(fg, cp[v], ig * gh);
+                cv[v] = cn;
+                hv[v] = og * tanh_approx(cn);
+            }
+            uint4 hp[2];
+            hp[0] = make_uint4(pack_bf16x2(hv[0], hv[1]), pack_bf16x2(hv[2], hv[3]),
+                               pack_bf16x2(hv[4], hv[5]), pack_bf16x2(hv[6], hv[7]));
+            hp[1] = make_uint4(pack_bf16x2(hv[8], hv[9]), pack_bf16x2(hv[10], hv[11]),
+                               pack_bf16x2(hv[12], hv[13]), pack_bf16x2(hv[14], hv[15]));
+            const long long hi = h_all_index(P, c, tl.axis, b, n);
+            uint4* hdst = reinterpret_cast<uint4*>(h_all + hi);
+            __stcg(hdst + 0, hp[0]);
+            __stcg(hdst + 1, hp[1]);
+            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n));
+#pragma unroll
+            for (int v = 0; v < 4; ++v)
+                __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
+            if (T.c_all) {
+                float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
+#pragma unroll
+                for (int v = 0; v < 4; ++v)
+                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+            }
+            if (top) {
+                uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n));
+                d[0] = hp[0];
+                d[1] = hp[1];
+            }
+            if (last) {
+                const long long ni = hn_index(P, c, tl.axis, b, n);
+                uint4* d = reinterpret_cast<uint4*>(h_n + ni);
+                d[0] = hp[0];
+                d[1] = hp[1];
+                float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
+#pragma unroll
+                for (int v = 0; v < 4; ++v)
+                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+            }
+            }  // valid
+        }
+        // publish this tile's share of the (cell, m-block) readiness counter
+        __threadfence();
+        named_bar_sync(1, 128);
+        if (warp == 2 && lane == 0)
+            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+        acc ^= 1;
+        if (acc == 0) acc_phase ^= 1;
+    }
+}
+
+__global__ void __launch_bounds__(THREADS, 1)
+wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
+                      const __grid_constant__ Maps M) {
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
+    uint8_t* smem = smem_raw + pad;
+    uint8_t* sA = smem;
+    uint8_t* sB = smem + STAGES * A_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE_BYTES);
+    uint64_t* full = bars;
+    uint64_t* empty = bars + STAGES;
+    uint64_t* tfull = bars + 2 * STAGES;
+    uint64_t* tempty = tfull + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull[a], 1);
+            mbar_init(&tempty[a], 4);
+        }
+        fence_mbarrier_init();
+        tma_prefetch_desc(&M.x);
+        tma_prefetch_desc(&M.ys);
+        tma_prefetch_desc(&M.h);
+        tma_prefetch_desc(&M.W);
+        tma_prefetch_desc(&M.U);
+    }
+    if (warp == 1) tmem_alloc(tmem_slot, TMEM_COLS);
+    tc_fence_before();
+    __syncthreads();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) run_producer(P, T, M, sA, sB, full, empty);
+    } else if (warp == 1) {
+        if (lane == 0) run_mma(P, tmem_base, sA, sB, full, empty, tfull, tempty);
+    } else {
+        run_epilogue(P, T, tmem_base, tfull, tempty);
+    }
+
+    tc_fence_before();
+    __syncthreads();
+    if (warp == 1) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, TMEM_COLS);
+    }
+}
+
+// ------------------------------------------------------------------------------ host side
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode_fn(std::string* err) {
+    static EncodeTiledFn fn = nullptr;
+    if (fn) return fn;
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
+    cudaError_t e = cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &ptr, 12000,
+                                                     cudaEnableDefault, &q);
+    if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !ptr) {
+        if (err) *err = "cuTensorMapEncodeTiled not available from the driver";
+        return nullptr;
+    }
+    fn = reinterpret_cast<EncodeTiledFn>(ptr);
+    return fn;
+}
+
+// Activation view (hidden, rows, batch) with a (64, 1, 128) box, 128-byte swizzle.
+bool encode_act(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, long long rows,
+                int B, std::string* err) {
+    const cuuint64_t dims[3] = {(cuuint64_t)H, (cuuint64_t)rows, (cuuint64_t)B};
+    const cuuint64_t strides[2] = {(cuuint64_t)H * 2, (cuuint64_t)rows * H * 2};
+    const cuuint32_t box[3] = {(cuuint32_t)BK, 1, (cuuint32_t)BM};
+    const cuuint32_t es[3] = {1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides,
+                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+        if (err) *err = "cuTensorMapEncodeTiled(activation) failed: " + std::to_string((int)r);
+        return false;
+    }
+    return true;
+}
+
+// Weight view (n, k, gate, slice) with a (64, 64, 4, 1) box, 128-byte swizzle: one box is the
+// [i | f | o | ĝ] x 64-unit N-tile of one 64-row K-chunk.
+bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int krows, int slices,
+               std::string* err) {
+    const cuuint64_t dims[4] = {(cuuint64_t)H, (cuuint64_t)krows, 4, (cuuint64_t)slices};
+    const cuuint64_t strides[3] = {(cuuint64_t)H * 2, (cuuint64_t)krows * H * 2,
+                                   (cuuint64_t)4 * krows * H * 2};
+    const cuuint32_t box[4] = {(cuuint32_t)BNU, (cuuint32_t)BK, 4, 1};
+    const cuuint32_t es[4] = {1, 1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides,
+                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+        if (err) *err = "cuTensorMapEncodeTiled(weight) failed: " + std::to_string((int)r);
+        return false;
+    }
+    return true;
+}
+
+}  // namespace
+
+cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
+                                  std::string* err) {
+    EncodeTiledFn enc = get_encode_fn(err);
+    if (!enc) return cudaErrorNotSupported;
+    Maps M;
+    const int slices = p.D * p.naxes;
+    if (!encode_act(enc, &M.x, t.x, p.H, p.L0, p.B, err)) return cudaErrorInvalidValue;
+    if (!encode_act(enc, &M.ys, p.kind == KIND_GRID ? t.ys : t.x, p.H,
+                    p.kind == KIND_GRID ? p.L1 : p.L0, p.B, err))
+        return cudaErrorInvalidValue;
+    if (!encode_act(enc, &M.h, t.h_all, p.H, h_rows(p), p.B, err)) return cudaErrorInvalidValue;
+    if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, err)) return cudaErrorInvalidValue;
+    if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, err)) return cudaErrorInvalidValue;
+
+    int dev = 0, nsm = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 SMEM_BYTES);
+    if (e != cudaSuccess) {
+        if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
+        return e;
+    }
+    long long grid = nsm;
+    if (grid > p.ntiles) grid = p.ntiles;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(THREADS);
+    cfg.dynamicSmemBytes = SMEM_BYTES;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeCooperative;
+    attr[0].val.cooperative = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel, p, t, M);
+    if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
+    return e;
+}
+
+}  // namespace ft

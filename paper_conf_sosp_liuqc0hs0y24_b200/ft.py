@@ -1,0 +1,247 @@
+"""Thin ctypes binding of libft.so (include/ft.h).  Argument marshalling only.
+
+Two layers:
+  * the raw C-ABI names (`ft_stacked_lstm_fwd`, `ft_dilated_rnn_fwd`, `ft_grid_rnn_fwd`, the
+    `*_workspace_size` queries, `ft_wavefront_cells`, ...) taking ints / raw pointers exactly
+    as the header declares them;
+  * torch-tensor conveniences (`stacked_lstm`, `dilated_rnn`, `grid_rnn`) that allocate the
+    outputs and the workspace with torch (PyTorch is plumbing: device memory and streams) and
+    call the raw entry point.  Every step of the computation runs in the library's kernels.
+
+There is no fallback: if libft.so is missing or a call fails, an exception is raised.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "libft.so")
+
+FT_OK, FT_ERR_INVALID_ARGUMENT, FT_ERR_UNSUPPORTED, FT_ERR_CUDA = 0, 1, 2, 3
+FT_ERR_WORKSPACE_TOO_SMALL = 5
+FT_F32, FT_BF16 = 0, 1
+FT_MAX_DEPTH = 64
+
+# every symbol include/ft.h declares (checked by tests/test_abi.py against the header)
+EXPORTS = (
+    "ft_version", "ft_status_string", "ft_last_error",
+    "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
+    "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
+    "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
+    "ft_wavefront_cells",
+)
+
+
+class FTError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{status_string(status)}: {msg}")
+        self.status = status
+
+
+_lib = None
+_c_int, _c_size, _c_vp, _c_ll = ctypes.c_int, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_longlong
+
+
+def lib():
+    """Load libft.so (in-tree).  Raises if it was not built — no CPU or library fallback."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_sosp_liuqc0hs0y24_b200.build`")
+        L = ctypes.CDLL(LIB_PATH)
+        L.ft_version.restype = _c_int
+        L.ft_status_string.restype = ctypes.c_char_p
+        L.ft_status_string.argtypes = [_c_int]
+        L.ft_last_error.restype = ctypes.c_char_p
+        L.ft_stacked_lstm_workspace_size.restype = _c_size
+        L.ft_stacked_lstm_workspace_size.argtypes = [_c_int] * 6
+        L.ft_dilated_rnn_workspace_size.restype = _c_size
+        L.ft_dilated_rnn_workspace_size.argtypes = [_c_int, _c_int, _c_int, _c_int, _c_vp, _c_int, _c_int]
+        L.ft_grid_rnn_workspace_size.restype = _c_size
+        L.ft_grid_rnn_workspace_size.argtypes = [_c_int] * 7
+        L.ft_stacked_lstm_fwd.restype = _c_int
+        L.ft_stacked_lstm_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 9 + [_c_vp, _c_size, _c_vp]
+        L.ft_dilated_rnn_fwd.restype = _c_int
+        L.ft_dilated_rnn_fwd.argtypes = [_c_int] * 4 + [_c_vp, _c_int] + [_c_vp] * 9 + [_c_vp, _c_size, _c_vp]
+        L.ft_grid_rnn_fwd.restype = _c_int
+        L.ft_grid_rnn_fwd.argtypes = [_c_int] * 6 + [_c_vp] * 10 + [_c_vp, _c_size, _c_vp]
+        L.ft_wavefront_cells.restype = _c_ll
+        L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
+        _lib = L
+    return _lib
+
+
+# ------------------------------------------------------------------------------ raw C ABI
+def ft_version() -> int:
+    return lib().ft_version()
+
+
+def status_string(s: int) -> str:
+    return lib().ft_status_string(s).decode()
+
+
+def ft_last_error() -> str:
+    return lib().ft_last_error().decode()
+
+
+def ft_stacked_lstm_workspace_size(batch, seq, hidden, depth, dt, h_all_provided):
+    return lib().ft_stacked_lstm_workspace_size(batch, seq, hidden, depth, dt, int(h_all_provided))
+
+
+def _int_array(vals):
+    arr = (ctypes.c_int * len(vals))(*[int(v) for v in vals])
+    return arr
+
+
+def ft_dilated_rnn_workspace_size(batch, seq, hidden, depth, dilations, dt, h_all_provided):
+    arr = _int_array(dilations) if dilations is not None else None
+    return lib().ft_dilated_rnn_workspace_size(batch, seq, hidden, depth,
+                                               ctypes.cast(arr, _c_vp) if arr is not None else None,
+                                               dt, int(h_all_provided))
+
+
+def ft_grid_rnn_workspace_size(batch, len_x, len_y, hidden, depth, dt, h_all_provided):
+    return lib().ft_grid_rnn_workspace_size(batch, len_x, len_y, hidden, depth, dt, int(h_all_provided))
+
+
+def ft_stacked_lstm_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n, c_n, h_all, c_all,
+                        workspace, workspace_bytes, stream) -> int:
+    return lib().ft_stacked_lstm_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n, c_n,
+                                     h_all, c_all, workspace, workspace_bytes, stream)
+
+
+def ft_dilated_rnn_fwd(batch, seq, hidden, depth, dilations, dt, x, W, U, b, y, h_n, c_n, h_all,
+                       c_all, workspace, workspace_bytes, stream) -> int:
+    arr = _int_array(dilations) if dilations is not None else None
+    return lib().ft_dilated_rnn_fwd(batch, seq, hidden, depth,
+                                    ctypes.cast(arr, _c_vp) if arr is not None else None, dt,
+                                    x, W, U, b, y, h_n, c_n, h_all, c_all, workspace,
+                                    workspace_bytes, stream)
+
+
+def ft_grid_rnn_fwd(batch, len_x, len_y, hidden, depth, dt, x, ys, W, U, b, out, h_n, c_n,
+                    h_all, c_all, workspace, workspace_bytes, stream) -> int:
+    return lib().ft_grid_rnn_fwd(batch, len_x, len_y, hidden, depth, dt, x, ys, W, U, b, out,
+                                 h_n, c_n, h_all, c_all, workspace, workspace_bytes, stream)
+
+
+def ft_wavefront_cells(kind, depth, len_a, len_b=1):
+    """Wavefront cell order as a list of (diagonal, d, i, j) — host only."""
+    n = lib().ft_wavefront_cells(kind, depth, len_a, len_b, None, 0)
+    if n < 0:
+        raise FTError(FT_ERR_INVALID_ARGUMENT, "bad schedule query")
+    buf = (ctypes.c_int * (4 * n))()
+    lib().ft_wavefront_cells(kind, depth, len_a, len_b, ctypes.cast(buf, _c_vp), n)
+    return [tuple(buf[4 * k:4 * k + 4]) for k in range(n)]
+
+
+def check(status: int):
+    if status != FT_OK:
+        raise FTError(status, ft_last_error())
+
+
+# ------------------------------------------------------------------------------ torch helpers
+def _torch():
+    import torch
+    return torch
+
+
+def _dt(t):
+    torch = _torch()
+    if t.dtype == torch.bfloat16:
+        return FT_BF16
+    if t.dtype == torch.float32:
+        return FT_F32
+    raise TypeError(f"unsupported dtype {t.dtype}")
+
+
+def _ptr(t):
+    return None if t is None else t.data_ptr()
+
+
+def _stream_ptr(stream):
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+class Workspace:
+    """A reusable device workspace (torch uint8 buffer) grown on demand."""
+
+    def __init__(self, device=None):
+        self.buf = None
+        self.device = device
+
+    def get(self, nbytes, device):
+        torch = _torch()
+        if self.buf is None or self.buf.numel() < nbytes or self.buf.device != device:
+            self.buf = torch.empty(max(nbytes, 256), dtype=torch.uint8, device=device)
+        return self.buf
+
+
+def stacked_lstm(x, W, U, b, want_all=False, dilations=None, stream=None, workspace=None, out=None):
+    """Stacked (or, with `dilations`, dilated) LSTM forward on the GPU through the C ABI.
+
+    x [B][T][H] (bf16 or fp32 CUDA tensor), W/U [D][4][H][H] (same dtype), b [D][4][H] fp32.
+    Returns dict y, h_n, c_n (+ h_all, c_all when want_all)."""
+    torch = _torch()
+    B, T, H = x.shape
+    D = W.shape[0]
+    dt = _dt(x)
+    dev = x.device
+    o = out or {}
+    y = o.get("y") if o.get("y") is not None else torch.empty((B, T, H), dtype=x.dtype, device=dev)
+    h_n = o.get("h_n") if o.get("h_n") is not None else torch.empty((B, D, H), dtype=x.dtype, device=dev)
+    c_n = o.get("c_n") if o.get("c_n") is not None else torch.empty((B, D, H), dtype=torch.float32, device=dev)
+    h_all = torch.empty((B, D, T, H), dtype=x.dtype, device=dev) if want_all else None
+    c_all = torch.empty((B, D, T, H), dtype=torch.float32, device=dev) if want_all else None
+    if dilations is None:
+        nbytes = ft_stacked_lstm_workspace_size(B, T, H, D, dt, h_all is not None)
+    else:
+        nbytes = ft_dilated_rnn_workspace_size(B, T, H, D, dilations, dt, h_all is not None)
+    ws = (workspace or Workspace()).get(nbytes, dev)
+    sp = _stream_ptr(stream)
+    if dilations is None:
+        st = ft_stacked_lstm_fwd(B, T, H, D, dt, _ptr(x), _ptr(W), _ptr(U), _ptr(b), _ptr(y),
+                                 _ptr(h_n), _ptr(c_n), _ptr(h_all), _ptr(c_all), ws.data_ptr(),
+                                 ws.numel(), sp)
+    else:
+        st = ft_dilated_rnn_fwd(B, T, H, D, dilations, dt, _ptr(x), _ptr(W), _ptr(U), _ptr(b),
+                                _ptr(y), _ptr(h_n), _ptr(c_n), _ptr(h_all), _ptr(c_all),
+                                ws.data_ptr(), ws.numel(), sp)
+    check(st)
+    r = dict(y=y, h_n=h_n, c_n=c_n)
+    if want_all:
+        r.update(h_all=h_all, c_all=c_all)
+    return r
+
+
+def dilated_rnn(x, W, U, b, dilations, **kw):
+    return stacked_lstm(x, W, U, b, dilations=list(dilations), **kw)
+
+
+def grid_rnn(x, ys, W, U, b, want_all=False, stream=None, workspace=None):
+    """Grid LSTM forward.  x [B][Lx][H], ys [B][Ly][H], W [D][2][4][H][H], U [D][2][4][2H][H],
+    b [D][2][4][H] fp32.  Returns dict out [B][Lx][Ly][2][H], h_n, c_n (+ h_all, c_all)."""
+    torch = _torch()
+    B, Lx, H = x.shape
+    Ly = ys.shape[1]
+    D = W.shape[0]
+    dt = _dt(x)
+    dev = x.device
+    out = torch.empty((B, Lx, Ly, 2, H), dtype=x.dtype, device=dev)
+    h_n = torch.empty((B, D, 2, H), dtype=x.dtype, device=dev)
+    c_n = torch.empty((B, D, 2, H), dtype=torch.float32, device=dev)
+    h_all = torch.empty((B, D, Lx, Ly, 2, H), dtype=x.dtype, device=dev) if want_all else None
+    c_all = torch.empty((B, D, Lx, Ly, 2, H), dtype=torch.float32, device=dev) if want_all else None
+    nbytes = ft_grid_rnn_workspace_size(B, Lx, Ly, H, D, dt, h_all is not None)
+    ws = (workspace or Workspace()).get(nbytes, dev)
+    st = ft_grid_rnn_fwd(B, Lx, Ly, H, D, dt, _ptr(x), _ptr(ys), _ptr(W), _ptr(U), _ptr(b),
+                         _ptr(out), _ptr(h_n), _ptr(c_n), _ptr(h_all), _ptr(c_all),
+                         ws.data_ptr(), ws.numel(), _stream_ptr(stream))
+    check(st)
+    r = dict(out=out, h_n=h_n, c_n=c_n)
+    if want_all:
+        r.update(h_all=h_all, c_all=c_all)
+    return r

@@ -1,0 +1,153 @@
+"""C-ABI contract tests that need no GPU: the library loads, exports every symbol include/ft.h
+declares, validates arguments before touching CUDA, sizes workspaces consistently, and its
+schedule enumerator (the same __host__ __device__ code the kernels run) is a legal wavefront
+(P10 on the product scheduler; region counts of §6.3)."""
+import ctypes
+import os
+import re
+
+import pytest
+
+from paper_conf_sosp_liuqc0hs0y24_b200 import build, ft
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    build.build()
+
+
+def _header_functions():
+    src = open(os.path.join(ROOT, "include", "ft.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(ft_[a-z0-9_]+)\s*\(", src)))
+
+
+def test_exports_every_header_symbol():
+    names = _header_functions()
+    assert len(names) >= 10
+    L = ctypes.CDLL(ft.LIB_PATH)
+    for n in names:
+        assert hasattr(L, n), f"libft.so does not export {n}"
+    assert sorted(ft.EXPORTS) == names
+
+
+def test_version_and_status_strings():
+    assert ft.ft_version() == 100
+    assert ft.status_string(ft.FT_OK) == "FT_OK"
+    assert ft.status_string(ft.FT_ERR_UNSUPPORTED) == "FT_ERR_UNSUPPORTED"
+    assert ft.status_string(ft.FT_ERR_WORKSPACE_TOO_SMALL) == "FT_ERR_WORKSPACE_TOO_SMALL"
+    assert ft.status_string(42) == "FT_ERR_UNKNOWN"
+
+
+FAKE = 1 << 20  # a 16-byte-aligned non-NULL "device" pointer; never dereferenced on error paths
+
+
+def _call(**over):
+    a = dict(batch=4, seq=8, hidden=64, depth=2, dt=ft.FT_BF16, x=FAKE, W=FAKE, U=FAKE, b=FAKE,
+             y=FAKE, h_n=FAKE, c_n=FAKE, h_all=None, c_all=None, workspace=FAKE,
+             workspace_bytes=1 << 40, stream=None)
+    a.update(over)
+    return ft.ft_stacked_lstm_fwd(**a)
+
+
+@pytest.mark.parametrize("over,code", [
+    (dict(batch=0), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(seq=-1), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(hidden=0), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(depth=0), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(dt=7), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(x=None), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(W=FAKE + 8), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(c_n=None), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(h_all=FAKE + 4), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(hidden=96), ft.FT_ERR_UNSUPPORTED),
+    (dict(depth=65), ft.FT_ERR_UNSUPPORTED),
+    (dict(workspace_bytes=16), ft.FT_ERR_WORKSPACE_TOO_SMALL),
+    (dict(workspace=None, workspace_bytes=0), ft.FT_ERR_INVALID_ARGUMENT),
+])
+def test_validation_before_any_launch(over, code):
+    assert _call(**over) == code
+    assert ft.ft_last_error()
+
+
+def test_dilation_and_grid_validation():
+    base = dict(batch=2, seq=4, hidden=64, depth=2, dt=ft.FT_BF16, x=FAKE, W=FAKE, U=FAKE, b=FAKE,
+                y=FAKE, h_n=FAKE, c_n=FAKE, h_all=None, c_all=None, workspace=FAKE,
+                workspace_bytes=1 << 40, stream=None)
+    assert ft.ft_dilated_rnn_fwd(dilations=[1, 0], **base) == ft.FT_ERR_INVALID_ARGUMENT
+    assert ft.ft_dilated_rnn_fwd(dilations=None, **base) == ft.FT_ERR_INVALID_ARGUMENT
+    g = dict(batch=2, len_x=3, len_y=3, hidden=64, depth=2, dt=ft.FT_BF16, x=FAKE, ys=None, W=FAKE,
+             U=FAKE, b=FAKE, out=FAKE, h_n=FAKE, c_n=FAKE, h_all=None, c_all=None, workspace=FAKE,
+             workspace_bytes=1 << 40, stream=None)
+    assert ft.ft_grid_rnn_fwd(**g) == ft.FT_ERR_INVALID_ARGUMENT
+    g.update(ys=FAKE, len_y=0)
+    assert ft.ft_grid_rnn_fwd(**g) == ft.FT_ERR_INVALID_ARGUMENT
+
+
+def test_valid_call_without_gpu_reports_cuda_error():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present: this checks the no-device error path")
+    assert _call() == ft.FT_ERR_CUDA
+
+
+def test_workspace_sizes():
+    B, T, H, D = 256, 100, 1024, 16
+    with_h = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_BF16, True)
+    without = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_BF16, False)
+    assert without - with_h >= B * D * T * H * 2  # the h_all SSA buffer lives in the workspace
+    assert with_h >= D * T * 2 * 4 + D * 2 * B * H * 4  # flags + 2-slot c ring
+    assert ft.ft_dilated_rnn_workspace_size(B, T, H, D, [1] * D, ft.FT_BF16, True) == with_h
+    big = ft.ft_dilated_rnn_workspace_size(B, T, H, D, [32] * D, ft.FT_BF16, True)
+    assert big > with_h  # ring of 2·s slots per layer
+    assert ft.ft_stacked_lstm_workspace_size(B, T, 96, D, ft.FT_BF16, True) == 0  # unsupported
+    assert ft.ft_grid_rnn_workspace_size(128, 32, 32, 512, 4, ft.FT_BF16, False) > 0
+
+
+# ----------------------------------------------------------------- product scheduler (P10)
+@pytest.mark.parametrize("D,T", [(2, 8), (16, 100), (8, 64), (1, 5), (5, 1), (3, 4)])
+def test_product_schedule_is_a_legal_wavefront(D, T):
+    cells = ft.ft_wavefront_cells(0, D, T)
+    assert len(cells) == D * T
+    seen = {}
+    for pos, (k, d, t, j) in enumerate(cells):
+        assert j == 0 and k == d + t
+        assert (d, t) not in seen
+        seen[(d, t)] = pos
+    diags = [k for k, _, _, _ in cells]
+    assert diags == sorted(diags) and len(set(diags)) == T + D - 1
+    for (d, t), pos in seen.items():  # producers (Table 4 e_depth, e_time) come earlier
+        if d > 0:
+            assert seen[(d - 1, t)] < pos
+        if t > 0:
+            assert seen[(d, t - 1)] < pos
+    # Table 5 (L355-L358): region_3 cells of diagonal j4 are exactly depth ∈ [max(1,j4-T+1), min(j4,D))
+    for j4 in range(2, T + D - 1):
+        got = sorted(d for k, d, t, _ in cells if k == j4 and d >= 1 and t >= 1)
+        assert got == list(range(max(1, j4 - T + 1), min(j4, D)))
+
+
+@pytest.mark.parametrize("D,Lx,Ly", [(4, 32, 32), (2, 3, 5), (3, 1, 4), (1, 2, 2)])
+def test_product_schedule_grid(D, Lx, Ly):
+    cells = ft.ft_wavefront_cells(1, D, Lx, Ly)
+    assert len(cells) == D * Lx * Ly
+    seen = {}
+    for pos, (k, d, i, j) in enumerate(cells):
+        assert k == d + i + j and (d, i, j) not in seen
+        seen[(d, i, j)] = pos
+    assert len({c[0] for c in cells}) == D + Lx + Ly - 2
+    for (d, i, j), pos in seen.items():
+        for dep in [(d - 1, i, j), (d, i - 1, j), (d, i, j - 1)]:
+            if min(dep) >= 0:
+                assert seen[dep] < pos
+
+
+def test_boundary_region_counts():
+    """§4.4 L243/L256 and §6.3: nested scans split into 2^(#scans) boundary regions —
+    4 block nodes for the stacked LSTM, 8 for the grid RNN.  A region = which producers exist."""
+    seq = {(d > 0, t > 0) for _, d, t, _ in ft.ft_wavefront_cells(0, 3, 4)}
+    assert len(seq) == 4
+    grid = {(d > 0, i > 0, j > 0) for _, d, i, j in ft.ft_wavefront_cells(1, 3, 3, 3)}
+    assert len(grid) == 8

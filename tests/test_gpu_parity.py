@@ -1,0 +1,198 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Tolerances (BASELINE.json north_star; reading R19 in DESIGN.md):
+  * fp32 path (SIMT, TF32 off):   max |gpu − oracle_f64| ≤ 1e-4 on every output tensor
+  * bf16 path (tcgen05):          normwise  max|gpu − ref| / max|ref| ≤ 2e-2 per output tensor
+Full-size configs (C3–C5) are checked on sampled batch rows: the batch `map` is independent
+(P6), so rows run alone through the oracle equal those rows of the full GPU run.
+"""
+import numpy as np
+import pytest
+import torch
+
+import ftgen
+import oracle
+from paper_conf_sosp_liuqc0hs0y24_b200 import build, ft
+
+pytestmark = pytest.mark.gpu
+
+F32_TOL = 1e-4
+BF16_TOL = 2e-2
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib(cuda_device):
+    build.build()
+    ft.lib()
+
+
+def dev(a, dtype):
+    t = torch.from_numpy(np.ascontiguousarray(a, dtype=np.float32))
+    return t.to(device="cuda", dtype=dtype)
+
+
+def host(t):
+    return t.float().cpu().numpy().astype(np.float64)
+
+
+def maxabs(a, b):
+    return float(np.max(np.abs(a - b))) if a.size else 0.0
+
+
+def normrel(a, ref):
+    den = float(np.max(np.abs(ref)))
+    return maxabs(a, ref) / max(den, 1e-30)
+
+
+def _check(got, ref, dtype, keys, rows=None, ctx=""):
+    for k in keys:
+        g = host(got[k])
+        if rows is not None:
+            g = g[rows]
+        r = ref[k]
+        assert g.shape == r.shape, (k, g.shape, r.shape)
+        assert np.all(np.isfinite(g)), f"{ctx} {k}: non-finite output"
+        if dtype == torch.float32:
+            err = maxabs(g, r)
+            assert err <= F32_TOL, f"{ctx} {k}: max abs err {err:.3e} > {F32_TOL}"
+        else:
+            err = normrel(g, r)
+            assert err <= BF16_TOL, f"{ctx} {k}: normwise rel err {err:.3e} > {BF16_TOL}"
+
+
+def _run_stacked(p, dtype, dil=None, want_all=False):
+    wd = dtype
+    x, W, U = dev(p["x"], wd), dev(p["W"], wd), dev(p["U"], wd)
+    b = dev(p["b"], torch.float32)
+    if dil is None:
+        r = ft.stacked_lstm(x, W, U, b, want_all=want_all)
+    else:
+        r = ft.dilated_rnn(x, W, U, b, dil, want_all=want_all)
+    torch.cuda.synchronize()
+    return r
+
+
+def _oracle_stacked(p, dil=None, want_all=False, rows=None):
+    x = p["x"] if rows is None else p["x"][rows]
+    if dil is None:
+        return oracle.stacked_lstm(x, p["W"], p["U"], p["b"], want_all=want_all)
+    return oracle.dilated_rnn(x, p["W"], p["U"], p["b"], dil, want_all=want_all)
+
+
+ALL = ("y", "h_n", "c_n", "h_all", "c_all")
+OUT = ("y", "h_n", "c_n")
+
+
+# ------------------------------------------------------------------------- fp32 path (BK1)
+def test_f32_C1_full():
+    c = ftgen.CONFIGS["C1"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C1"), "f32")
+    got = _run_stacked(p, torch.float32, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.float32, ALL, ctx="C1")
+
+
+@pytest.mark.parametrize("B,T,H,D", [(1, 1, 8, 1), (3, 5, 33, 2), (33, 4, 16, 3), (2, 9, 64, 4),
+                                     (70, 3, 40, 2)])
+def test_f32_edge_shapes(B, T, H, D):
+    p = ftgen.stacked_inputs(B, T, H, D, 101 + B + T, "f32", scale=2.0)
+    got = _run_stacked(p, torch.float32, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.float32, ALL, ctx=f"f32 {B,T,H,D}")
+
+
+@pytest.mark.parametrize("dil", [[1, 2, 3], [4, 1, 9], [2, 2, 2]])
+def test_f32_dilated(dil):
+    p = ftgen.stacked_inputs(5, 11, 24, len(dil), 55, "f32", scale=2.0)
+    got = _run_stacked(p, torch.float32, dil=dil, want_all=True)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.float32, ALL, ctx=f"dil {dil}")
+
+
+@pytest.mark.parametrize("B,Lx,Ly,H,D", [(3, 3, 4, 16, 2), (1, 1, 5, 8, 3), (34, 4, 1, 32, 2)])
+def test_f32_grid(B, Lx, Ly, H, D):
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, 77, "f32", scale=2.0)
+    args = [dev(g[k], torch.float32) for k in ("x", "ys", "W", "U", "b")]
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.float32, ("out", "h_n", "c_n", "h_all", "c_all"), ctx="f32 grid")
+
+
+# ------------------------------------------------------------------------- bf16 tcgen05 path
+@pytest.mark.parametrize("B,T,H,D", [(1, 1, 64, 1), (4, 3, 64, 2), (130, 3, 128, 2),
+                                     (5, 9, 192, 3), (256, 4, 256, 2)])
+def test_bf16_small_and_ragged(B, T, H, D):
+    p = ftgen.stacked_inputs(B, T, H, D, 202 + B, "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"bf16 {B,T,H,D}")
+
+
+def test_bf16_C2_full():
+    c = ftgen.CONFIGS["C2"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C2"), "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="C2")
+
+
+def test_bf16_signal_preserving_scale():
+    """The second input set of DESIGN.md (U(±2/√H)): deeper layers carry more signal."""
+    p = ftgen.stacked_inputs(64, 16, 256, 4, 303, "bf16", scale=2.0)
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="scale2")
+
+
+@pytest.mark.parametrize("dil", [[1, 2, 4], [3, 1, 7], [8, 8]])
+def test_bf16_dilated_small(dil):
+    p = ftgen.stacked_inputs(20, 13, 128, len(dil), 404, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"dil {dil}")
+
+
+@pytest.mark.parametrize("B,Lx,Ly,H,D", [(3, 3, 4, 64, 2), (130, 2, 3, 128, 2), (8, 1, 6, 64, 3)])
+def test_bf16_grid_small(B, Lx, Ly, H, D):
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, 505, "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx="bf16 grid")
+
+
+def test_bf16_deterministic():
+    p = ftgen.stacked_inputs(130, 7, 128, 3, 606, "bf16")
+    a = _run_stacked(p, torch.bfloat16, want_all=True)
+    b = _run_stacked(p, torch.bfloat16, want_all=True)
+    for k in ALL:
+        assert torch.equal(a[k], b[k]), k
+
+
+# ------------------------------------------------------------------------- full sizes, sampled
+@pytest.mark.slow
+def test_bf16_C3_sampled_rows():
+    c = ftgen.CONFIGS["C3"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C3"), "bf16")
+    got = _run_stacked(p, torch.bfloat16)
+    rows = ftgen.sample_rows(c["batch"], 0, 1)[:4]
+    ref = _oracle_stacked(p, rows=rows)
+    _check(got, ref, torch.bfloat16, OUT, rows=rows, ctx="C3")
+
+
+@pytest.mark.slow
+def test_bf16_C4_sampled_rows():
+    c = ftgen.CONFIGS["C4"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C4"), "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=list(c["dilations"]))
+    rows = ftgen.sample_rows(c["batch"], 2, 2)
+    ref = _oracle_stacked(p, dil=list(c["dilations"]), rows=rows)
+    _check(got, ref, torch.bfloat16, OUT, rows=rows, ctx="C4")
+
+
+@pytest.mark.slow
+def test_bf16_C5_sampled_rows():
+    c = ftgen.CONFIGS["C5"]
+    g = ftgen.grid_inputs(c["batch"], c["len_x"], c["len_y"], c["hidden"], c["depth"],
+                          ftgen.config_seed("C5"), "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    got = ft.grid_rnn(*args)
+    torch.cuda.synchronize()
+    rows = ftgen.sample_rows(c["batch"], 0, 3)[:4]
+    ref = oracle.grid_rnn(g["x"][rows], g["ys"][rows], g["W"], g["U"], g["b"])
+    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n"), rows=rows, ctx="C5")
