@@ -1,0 +1,38 @@
+"""Quick device timing of the forward (development aid; bench.py is the contract)."""
+import sys, time, json
+import numpy as np, torch
+sys.path.insert(0, ".")
+import ftgen
+from paper_conf_sosp_liuqc0hs0y24_b200 import ft
+
+def timeit(fn, reps=10, warm=3):
+    for _ in range(warm): fn()
+    torch.cuda.synchronize()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for _ in range(reps):
+        s.record(); fn(); e.record(); torch.cuda.synchronize(); ts.append(s.elapsed_time(e))
+    return float(np.median(ts)), float(np.min(ts))
+
+res = {}
+for name in sys.argv[1:] or ["C2", "C3", "C4", "C5"]:
+    c = ftgen.CONFIGS[name]
+    ws = ft.Workspace()
+    if c["kind"] == "grid":
+        g = ftgen.grid_inputs(c["batch"], c["len_x"], c["len_y"], c["hidden"], c["depth"], 1, "bf16")
+        a = [torch.from_numpy(g[k]).cuda().to(torch.bfloat16) for k in ("x","ys","W","U")] + [torch.from_numpy(g["b"]).cuda()]
+        fn = lambda: ft.grid_rnn(*a, workspace=ws)
+        flops = 48 * c["hidden"]**2 * c["len_x"] * c["len_y"] * c["depth"] * c["batch"]
+    else:
+        p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], 1, "bf16")
+        a = [torch.from_numpy(p[k]).cuda().to(torch.bfloat16) for k in ("x","W","U")] + [torch.from_numpy(p["b"]).cuda()]
+        dil = list(c.get("dilations", [])) or None
+        fn = lambda: ft.stacked_lstm(*a, dilations=dil, workspace=ws)
+        H, T, D, B = c["hidden"], c["seq"], c["depth"], c["batch"]
+        if dil:
+            flops = sum(2*B*4*H*(H*T + H*max(0, T-s)) for s in dil)
+        else:
+            flops = 16 * H * H * T * D * B
+    med, mn = timeit(fn)
+    res[name] = dict(ms_median=med, ms_min=mn, tflops=flops / med / 1e9, seq_per_s=c["batch"] / med * 1e3)
+    print(name, json.dumps(res[name]), flush=True)
