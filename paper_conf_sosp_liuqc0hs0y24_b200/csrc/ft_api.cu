@@ -219,6 +219,80 @@ FT_API ft_status ft_stacked_lstm_fwd(int batch, int seq, int hidden, int depth, 
                    workspace, workspace_bytes, stream);
 }
 
+namespace {
+struct HostIoPlan {
+    size_t x_off, y_off, hn_off, cn_off, inner_off, total;
+};
+HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, size_t inner) {
+    const size_t es = elem_size(dt);
+    HostIoPlan h{};
+    h.x_off = 0;
+    h.y_off = round_up((size_t)batch * seq * hidden * es, 256);
+    h.hn_off = h.y_off + round_up((size_t)batch * seq * hidden * es, 256);
+    h.cn_off = h.hn_off + round_up((size_t)batch * depth * hidden * es, 256);
+    h.inner_off = h.cn_off + round_up((size_t)batch * depth * hidden * 4, 256);
+    h.total = h.inner_off + inner;
+    return h;
+}
+}  // namespace
+
+FT_API size_t ft_stacked_lstm_hostio_workspace_size(int batch, int seq, int hidden, int depth,
+                                                    ft_dtype dt) {
+    const size_t inner = ft_stacked_lstm_workspace_size(batch, seq, hidden, depth, dt, 0);
+    if (inner == 0) return 0;
+    return plan_hostio(batch, seq, hidden, depth, dt, inner).total;
+}
+
+FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt,
+                                            const void* x_host, const void* W, const void* U,
+                                            const float* b, void* y_host, void* h_n_host,
+                                            float* c_n_host, void* workspace,
+                                            size_t workspace_bytes, void* stream) {
+    if (depth <= 0) return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    if (depth > FT_MAX_DEPTH) return fail(FT_ERR_UNSUPPORTED, "depth > FT_MAX_DEPTH");
+    int ones[FT_MAX_DEPTH];
+    for (int d = 0; d < depth; ++d) ones[d] = 1;
+    ft::Problem p;
+    ft_status st = make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, ones, dt, &p);
+    if (st != FT_OK) return st;
+    if (!x_host || !y_host || !h_n_host || !c_n_host)
+        return fail(FT_ERR_INVALID_ARGUMENT, "a host buffer is NULL");
+    REQUIRE_PTR(W, "W");
+    REQUIRE_PTR(U, "U");
+    REQUIRE_PTR(b, "b");
+    const size_t inner = ft_stacked_lstm_workspace_size(batch, seq, hidden, depth, dt, 0);
+    const HostIoPlan hp = plan_hostio(batch, seq, hidden, depth, dt, inner);
+    if (!workspace) return fail(FT_ERR_INVALID_ARGUMENT, "workspace is NULL");
+    if (!aligned16(workspace)) return fail(FT_ERR_INVALID_ARGUMENT, "workspace not 16-byte aligned");
+    if (workspace_bytes < hp.total)
+        return fail(FT_ERR_WORKSPACE_TOO_SMALL, "workspace_bytes " + std::to_string(workspace_bytes) +
+                                                    " < required " + std::to_string(hp.total));
+    st = check_device();
+    if (st != FT_OK) return st;
+    uint8_t* ws = static_cast<uint8_t*>(workspace);
+    cudaStream_t s = static_cast<cudaStream_t>(stream);
+    const size_t es = elem_size(dt);
+    const size_t xb = (size_t)batch * seq * hidden * es, hb = (size_t)batch * depth * hidden * es;
+    const size_t cb = (size_t)batch * depth * hidden * 4;
+    cudaError_t e = cudaMemcpyAsync(ws + hp.x_off, x_host, xb, cudaMemcpyHostToDevice, s);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("x H2D: ") + cudaGetErrorString(e));
+    ft::Tensors t;
+    t.x = ws + hp.x_off;
+    t.W = W;
+    t.U = U;
+    t.b = b;
+    t.y = ws + hp.y_off;
+    t.h_n = ws + hp.hn_off;
+    t.c_n = reinterpret_cast<float*>(ws + hp.cn_off);
+    st = run(p, dt, t, ws + hp.inner_off, inner, stream);
+    if (st != FT_OK) return st;
+    e = cudaMemcpyAsync(y_host, ws + hp.y_off, xb, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(h_n_host, ws + hp.hn_off, hb, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("D2H: ") + cudaGetErrorString(e));
+    return FT_OK;
+}
+
 FT_API size_t ft_dilated_rnn_workspace_size(int batch, int seq, int hidden, int depth,
                                             const int* dilations, ft_dtype dt, int h_all_provided) {
     ft::Problem p;

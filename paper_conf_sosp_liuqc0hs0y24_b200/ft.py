@@ -27,6 +27,7 @@ FT_MAX_DEPTH = 64
 EXPORTS = (
     "ft_version", "ft_status_string", "ft_last_error",
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
+    "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells",
@@ -66,6 +67,10 @@ def lib():
         L.ft_dilated_rnn_fwd.argtypes = [_c_int] * 4 + [_c_vp, _c_int] + [_c_vp] * 9 + [_c_vp, _c_size, _c_vp]
         L.ft_grid_rnn_fwd.restype = _c_int
         L.ft_grid_rnn_fwd.argtypes = [_c_int] * 6 + [_c_vp] * 10 + [_c_vp, _c_size, _c_vp]
+        L.ft_stacked_lstm_hostio_workspace_size.restype = _c_size
+        L.ft_stacked_lstm_hostio_workspace_size.argtypes = [_c_int] * 5
+        L.ft_stacked_lstm_fwd_hostio.restype = _c_int
+        L.ft_stacked_lstm_fwd_hostio.argtypes = [_c_int] * 5 + [_c_vp] * 7 + [_c_vp, _c_size, _c_vp]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         _lib = L
@@ -109,6 +114,17 @@ def ft_stacked_lstm_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n, c_n, 
                         workspace, workspace_bytes, stream) -> int:
     return lib().ft_stacked_lstm_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n, c_n,
                                      h_all, c_all, workspace, workspace_bytes, stream)
+
+
+def ft_stacked_lstm_hostio_workspace_size(batch, seq, hidden, depth, dt):
+    return lib().ft_stacked_lstm_hostio_workspace_size(batch, seq, hidden, depth, dt)
+
+
+def ft_stacked_lstm_fwd_hostio(batch, seq, hidden, depth, dt, x_host, W, U, b, y_host, h_n_host,
+                               c_n_host, workspace, workspace_bytes, stream) -> int:
+    return lib().ft_stacked_lstm_fwd_hostio(batch, seq, hidden, depth, dt, x_host, W, U, b,
+                                            y_host, h_n_host, c_n_host, workspace,
+                                            workspace_bytes, stream)
 
 
 def ft_dilated_rnn_fwd(batch, seq, hidden, depth, dilations, dt, x, W, U, b, y, h_n, c_n, h_all,
