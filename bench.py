@@ -65,7 +65,7 @@ def load_peaks():
 
 def load_traffic():
     """dram read+write bytes per launch from the committed ncu --set full summary, or None."""
-    p = os.path.join(ROOT, "profiles", "ncu_C3_summary.json")
+    p = os.path.join(ROOT, "profiles", "latest_C3_ncu_summary.json")
     if os.path.exists(p):
         with open(p) as f:
             d = json.load(f)
