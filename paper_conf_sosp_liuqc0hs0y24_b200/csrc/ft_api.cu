@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -54,7 +55,13 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
     p->L0 = L0;
     p->L1 = L1;
     p->naxes = (kind == ft::KIND_SEQ) ? 1 : 2;
-    p->BM = dt == FT_BF16 ? ft::BF16_BM : ft::F32_BM;
+    // bf16: one tcgen05 tile covers 128 batch rows (1 CTA) or 256 (a CTA pair, cta_group::2)
+    p->BM = dt == FT_BF16 ? (B > ft::BF16_BM ? 2 * ft::BF16_BM : ft::BF16_BM) : ft::F32_BM;
+    p->flag_mult = dt == FT_BF16 ? p->BM / ft::BF16_BM : 1;
+    {
+        const char* env = getenv("FT_L2_RESIDENT_LAYERS");
+        p->resident_layers = env ? atoi(env) : 0;
+    }
     p->BNU = dt == FT_BF16 ? ft::BF16_BNU : ft::F32_BNU;
     p->MB = (B + p->BM - 1) / p->BM;
     p->NT = (H + p->BNU - 1) / p->BNU;

@@ -32,6 +32,8 @@ struct Problem {
     int naxes;           // 1 (seq) or 2 (grid)
     int BM, BNU;         // batch rows and hidden units per tile (kernel-specific)
     int MB, NT;          // m-blocks = ceil(B/BM), n-tiles per axis = ceil(H/BNU)
+    int flag_mult;       // counter increments per tile (CTAs per tile: 2 for a tcgen05 CTA pair)
+    int resident_layers; // bf16: layers whose weights are kept in L2 (evict_last); others stream
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT
     int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)
@@ -100,8 +102,8 @@ FT_HD long long cell_lin(const Problem& p, int d, int i, int j) {
 
 FT_HD int tiles_per_cell(const Problem& p) { return p.naxes * p.MB * p.NT; }
 
-// Flags: one int per (cell, m-block); complete when it reaches naxes * NT.
-FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT; }
+// Flags: one int per (cell, m-block); complete when it reaches naxes * NT * flag_mult.
+FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
 
 // Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).
 struct Cursor {

@@ -1,32 +1,41 @@
 // wavefront_bf16.cu — BK2/BK3/BK4: the persistent sm_100a wavefront (stacked, dilated, grid).
 //
-// One launch runs the whole nest.  Every CTA (one per SM, cooperative launch so all are
-// co-resident) walks the global tile sequence in wavefront order (ft_common.cuh) with stride
-// gridDim.x.  A tile = (cell, axis, 128 batch rows, 64 hidden units x 4 gates):
+// One launch runs the whole nest.  Every CTA (one per SM; all co-resident) walks the global tile
+// sequence in wavefront order (ft_common.cuh).  A tile = (cell, axis, M batch rows, 64 hidden
+// units x 4 gates):
 //
-//   z[128 x 256] = Σ_seg A_seg[128 x H] · B_seg[H x 256] + b          (Listing 2)
+//   z[M x 256] = Σ_seg A_seg[M x H] · B_seg[H x 256] + b          (Listing 2)
 //
 // the horizontal merge of the 4 gate maps (N = 4 x 64, L287) and the vertical merge of
-// x@w + h@u (K = segments x H, L289–L293) as one tcgen05 GEMM; A = activation rows (batch =
-// the GEMM M dimension, the reuse dimension of L345–L349), B = the weight slice W[d][g][k][n]
-// used as an MN-major operand (n contiguous, no repacking).  The pointwise LSTM update
-// (L611–L615) runs in the epilogue straight out of TMEM.
+// x@w + h@u (K = segments x H, L289–L293) as one tcgen05 GEMM; A = activation rows (batch = the
+// GEMM M dimension — the reuse dimension of L345–L349), B = the weight slice W[d][g][k][n] used
+// as an MN-major operand (n contiguous, no repacking).  The LSTM update (L611–L615) runs in the
+// epilogue straight out of TMEM.
 //
-// Warp roles (192 threads):
-//   warp 0      TMA producer: waits the tile's producer cells (readiness flags), then streams
-//               K-chunks of A (128 rows x 64 k, 16 KiB) and B (4 gates x 64 k x 64 n, 32 KiB)
-//               into a 4-stage shared-memory ring (mbarrier full/empty).
-//   warp 1      MMA issuer: one thread issues tcgen05.mma (M128 N256 K16) into a TMEM
-//               accumulator, double-buffered (2 x 256 columns) so tile n+1's MMAs overlap
-//               tile n's epilogue.
-//   warps 2-5   epilogue: tcgen05.ld → +b, σ/σ/σ/tanh, c' = f·c + i·ĝ, h' = o·tanh(c')
-//               (fp32 registers), h' → bf16 → h_all (the SSA buffer node, L217) and y / h_n;
-//               c' → fp32 cell-state ring (+ c_all / c_n); then release the tile's share of the
+// Two instantiations:
+//   CG = 1  one CTA per tile, M = 128 (batch <= 128)
+//   CG = 2  a CTA pair (cluster of 2, tcgen05 cta_group::2) per tile, M = 256: each CTA stages its
+//           128 A rows and HALF of the N = 256 weight columns (gates i,f or o,ĝ); the leader CTA
+//           issues M256 N256 K16 MMAs reading both CTAs' shared memory, so each weight tile is
+//           fetched once per cell for the whole 256-row batch and per-CTA weight traffic halves.
+//
+// Warp roles (192 threads per CTA):
+//   warp 0      TMA producer: waits the tile's producer cells (readiness counters), then streams
+//               64-deep K-chunks of A and B into a STAGES-deep shared-memory ring (mbarriers).
+//   warp 1      MMA issuer (leader CTA): one thread issues tcgen05.mma into a double-buffered
+//               TMEM accumulator (2 x 256 fp32 columns) so tile n+1's MMAs overlap tile n's
+//               epilogue.
+//   warps 2-5   epilogue: tcgen05.ld → +b, σ/σ/σ/tanh, c' = f·c + i·ĝ, h' = o·tanh(c') in fp32
+//               registers; h' → bf16 → h_all (the SSA buffer node, L217) and y / h_n; c' → fp32
+//               cell-state ring (+ c_all / c_n); then release the tile's share of the
 //               (cell, m-block) readiness counter.
 //
 // Cross-CTA ordering (generic-proxy stores → another SM's async-proxy TMA loads):
 //   writer: st.global …; fence.acq_rel.gpu (every thread); bar.sync; red.release.gpu
 //   reader: ld.acquire.gpu (bounded spin); fence.proxy.async.global; cp.async.bulk.tensor
+// L2 policy: streamed weights EVICT_FIRST (they are re-read only one diagonal later, after the
+// whole 256 MiB weight set went through L2), weights of the first `resident_layers` layers
+// EVICT_LAST (kept in L2 across time steps — the reuse of L345–L349), activations EVICT_NORMAL.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -42,34 +51,49 @@ namespace {
 
 using namespace sm100;
 
-constexpr int BM = BF16_BM;    // 128 batch rows = TMEM lanes = UMMA M
+constexpr int ROWS = BF16_BM;  // 128 batch rows per CTA = TMEM lanes
 constexpr int BNU = BF16_BNU;  // 64 hidden units per tile
 constexpr int BN = 4 * BNU;    // 256 = UMMA N (i | f | o | ĝ)
 constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16
 constexpr int UK = 16;         // UMMA K for kind::f16
-constexpr int STAGES = 4;
-constexpr int A_BYTES = BM * BK * 2;  // 16 KiB
-constexpr int B_BYTES = BN * BK * 2;  // 32 KiB
-constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
 constexpr int THREADS = 192;
 constexpr int TMEM_COLS = 2 * BN;  // double-buffered accumulator
-constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024;
-constexpr uint32_t IDESC = make_idesc_bf16_f32(BM, BN, /*a MN-major*/ false, /*b MN-major*/ true);
+
+template <int CG>
+struct KCfg {
+    static constexpr int GATES = 4 / CG;                       // weight gate boxes per CTA
+    static constexpr int A_BYTES = ROWS * BK * 2;              // 16 KiB
+    static constexpr int B_BYTES = GATES * BNU * BK * 2;       // 32 KiB (CG 1) / 16 KiB (CG 2)
+    static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+    static constexpr int STAGES = CG == 1 ? 4 : 6;
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024;
+    static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
+};
 
 struct Maps {
     CUtensorMap x, ys, h, W, U;
 };
 
+__device__ __forceinline__ int weight_layer(const Problem& P, int slice) {
+    return P.kind == KIND_SEQ ? slice : slice >> 1;
+}
+
 // ------------------------------------------------------------------------------ producer
+template <int CG>
 __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
                                              uint8_t* sA, uint8_t* sB, uint64_t* full,
-                                             uint64_t* empty) {
+                                             uint64_t* empty, uint32_t rank) {
+    using C = KCfg<CG>;
     int stage = 0;
     uint32_t phase = 0;
     Cursor cur = cursor_begin();
     const int target = flag_target(P);
     const int kchunks = P.H / BK;
-    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+    const uint64_t pol_stream = policy_evict_first();
+    const uint64_t pol_keep = policy_evict_last();
+    const uint64_t pol_act = policy_evict_normal();
+    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
         long long prod[3];
         const int np = producers(P, tl.cell, prod);
@@ -77,16 +101,22 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         fence_proxy_async_global();
         Segment seg[3];
         const int ns = segments(P, tl, seg);
+        const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
         for (int s = 0; s < ns; ++s) {
             const CUtensorMap* am = seg[s].src == SRC_X ? &M.x : (seg[s].src == SRC_YS ? &M.ys : &M.h);
             const CUtensorMap* bm = seg[s].wsel == W_IN ? &M.W : &M.U;
+            const uint64_t wpol = weight_layer(P, seg[s].slice) < P.resident_layers ? pol_keep : pol_stream;
             for (int kc = 0; kc < kchunks; ++kc) {
                 mbar_wait(&empty[stage], phase ^ 1);
-                mbar_arrive_expect_tx(&full[stage], STAGE_BYTES);
-                tma_load_3d(sA + stage * A_BYTES, am, &full[stage], kc * BK, seg[s].row, tl.m * BM);
-                tma_load_4d(sB + stage * B_BYTES, bm, &full[stage], tl.n * BNU,
-                            seg[s].krow0 + kc * BK, 0, seg[s].slice);
-                if (++stage == STAGES) {
+                uint32_t bar = smem_u32(&full[stage]);
+                if constexpr (CG == 2) bar = mapa_shared(bar, 0);  // the leader's barrier
+                if (rank == 0) mbar_arrive_expect_tx(&full[stage], CG * C::STAGE_BYTES);
+                tma_load_3d_hint<CG>(sA + stage * C::A_BYTES, am, bar, kc * BK, seg[s].row, arow0,
+                                     pol_act);
+                tma_load_4d_hint<CG>(sB + stage * C::B_BYTES, bm, bar, tl.n * BNU,
+                                     seg[s].krow0 + kc * BK, (int)rank * C::GATES, seg[s].slice,
+                                     wpol);
+                if (++stage == C::STAGES) {
                     stage = 0;
                     phase ^= 1;
                 }
@@ -96,16 +126,19 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
 }
 
 // ------------------------------------------------------------------------------ MMA issuer
+template <int CG>
 __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, uint8_t* sA,
                                         uint8_t* sB, uint64_t* full, uint64_t* empty,
                                         uint64_t* tfull, uint64_t* tempty) {
+    using C = KCfg<CG>;
     int stage = 0;
     uint32_t phase = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
     Cursor cur = cursor_begin();
     const int kchunks = P.H / BK;
-    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
         Segment seg[3];
         const int nchunks = segments(P, tl, seg) * kchunks;
@@ -115,22 +148,22 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
         for (int c = 0; c < nchunks; ++c) {
             mbar_wait(&full[stage], phase);
             tc_fence_after();
-            // A: K-major, SW128: rows of 128 B, 8-row groups 1024 B apart (SBO); K step = +32 B.
-            // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups
-            //    1024 B apart (SBO); K step of 16 rows = +2048 B.
-            const uint64_t ad = make_sdesc(smem_u32(sA + stage * A_BYTES), 16, 1024);
-            const uint64_t bd = make_sdesc(smem_u32(sB + stage * B_BYTES), 8192, 1024);
+            // A: K-major, SW128: 128-B rows, 8-row groups 1024 B apart (SBO); K step = +32 B.
+            // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups 1024 B
+            //    apart (SBO); K step of 16 rows = +2048 B.  CG 2: each CTA holds half the atoms.
+            const uint64_t ad = make_sdesc(smem_u32(sA + stage * C::A_BYTES), 16, 1024);
+            const uint64_t bd = make_sdesc(smem_u32(sB + stage * C::B_BYTES), 8192, 1024);
 #pragma unroll
             for (int kk = 0; kk < BK / UK; ++kk)
-                umma_f16(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
-                         bd + (uint64_t)((kk * UK * 128) >> 4), IDESC, (c | kk) != 0);
-            umma_commit(&empty[stage]);
-            if (++stage == STAGES) {
+                umma_f16_cg<CG>(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
+                                bd + (uint64_t)((kk * UK * 128) >> 4), C::IDESC, (c | kk) != 0);
+            umma_commit_cg<CG>(&empty[stage]);
+            if (++stage == C::STAGES) {
                 stage = 0;
                 phase ^= 1;
             }
         }
-        umma_commit(&tfull[acc]);
+        umma_commit_cg<CG>(&tfull[acc]);
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
@@ -142,8 +175,21 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
     return *reinterpret_cast<uint32_t*>(&v);
 }
 
+__device__ __forceinline__ void load16(const float* src, float (&v)[16]) {
+    const float4* s4 = reinterpret_cast<const float4*>(src);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        const float4 t = __ldg(s4 + q);
+        v[4 * q + 0] = t.x;
+        v[4 * q + 1] = t.y;
+        v[4 * q + 2] = t.z;
+        v[4 * q + 3] = t.w;
+    }
+}
+
+template <int CG>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
-                                             uint64_t* tfull, uint64_t* tempty) {
+                                             uint64_t* tfull, uint64_t* tempty, uint32_t rank) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3;  // TMEM lane quadrant this warp may access
     const int row = q * 32 + lane;
@@ -154,7 +200,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
     __nv_bfloat16* y = (__nv_bfloat16*)T.y;
     __nv_bfloat16* h_n = (__nv_bfloat16*)T.h_n;
-    for (long long tile = blockIdx.x; tile < P.ntiles; tile += gridDim.x) {
+    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
         const Cell c = tl.cell;
         int ci = 0, cj = 0;
@@ -163,7 +210,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         mbar_wait(&tfull[acc], acc_phase);
         tc_fence_after();
 
-        const int b = tl.m * BM + row;
+        const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
         const int slice = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
         const float* bias = T.b + (long long)slice * 4 * P.H;
@@ -181,72 +228,85 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             if (u0 + 16 == BNU) {  // accumulator buffer drained → hand it back to the MMA warp
                 tc_fence_before();
                 __syncwarp();
-                if (lane == 0) mbar_arrive(&tempty[acc]);
+                if (lane == 0) {
+                    if constexpr (CG == 1)
+                        mbar_arrive(&tempty[acc]);
+                    else
+                        mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[acc]), 0));
+                }
             }
             if (valid) {
-            const int n = tl.n * BNU + u0;
-            float cp[16];
-            if (cprod >= 0) {
-                const float4* src = reinterpret_cast<const float4*>(
-                    T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n));
+                const int n = tl.n * BNU + u0;
+                float cp[16];
+                if (cprod >= 0) {
+                    const float4* src = reinterpret_cast<const float4*>(
+                        T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n));
 #pragma unroll
-                for (int v = 0; v < 4; ++v) {
-                    const float4 t4 = __ldcg(src + v);
-                    cp[4 * v + 0] = t4.x; cp[4 * v + 1] = t4.y;
-                    cp[4 * v + 2] = t4.z; cp[4 * v + 3] = t4.w;
+                    for (int v = 0; v < 4; ++v) {
+                        const float4 t4 = __ldcg(src + v);
+                        cp[4 * v + 0] = t4.x;
+                        cp[4 * v + 1] = t4.y;
+                        cp[4 * v + 2] = t4.z;
+                        cp[4 * v + 3] = t4.w;
+                    }
+                } else {
+#pragma unroll
+                    for (int v = 0; v < 16; ++v) cp[v] = 0.f;
                 }
-            } else {
+                float bi[16], bf[16], bo[16], bg[16];
+                load16(bias + 0 * P.H + n, bi);
+                load16(bias + 1 * P.H + n, bf);
+                load16(bias + 2 * P.H + n, bo);
+                load16(bias + 3 * P.H + n, bg);
+                float hv[16], cv[16];
 #pragma unroll
-                for (int v = 0; v < 16; ++v) cp[v] = 0.f;
-            }
-            float hv[16], cv[16];
-#pragma unroll
-            for (int v = 0; v < 16; ++v) {
-                const float ig = sigmoid_approx(zi[v] + __ldg(bias + 0 * P.H + n + v));
-                const float fg = sigmoid_approx(zf[v] + __ldg(bias + 1 * P.H + n + v));
-                const float og = sigmoid_approx(zo[v] + __ldg(bias + 2 * P.H + n + v));
-                const float gh = tanh_approx(zg[v] + __ldg(bias + 3 * P.H + n + v));
-                const float cn = fmaf(fg, cp[v], ig * gh);
-                cv[v] = cn;
-                hv[v] = og * tanh_approx(cn);
-            }
-            uint4 hp[2];
-            hp[0] = make_uint4(pack_bf16x2(hv[0], hv[1]), pack_bf16x2(hv[2], hv[3]),
-                               pack_bf16x2(hv[4], hv[5]), pack_bf16x2(hv[6], hv[7]));
-            hp[1] = make_uint4(pack_bf16x2(hv[8], hv[9]), pack_bf16x2(hv[10], hv[11]),
-                               pack_bf16x2(hv[12], hv[13]), pack_bf16x2(hv[14], hv[15]));
-            const long long hi = h_all_index(P, c, tl.axis, b, n);
-            uint4* hdst = reinterpret_cast<uint4*>(h_all + hi);
-            __stcg(hdst + 0, hp[0]);
-            __stcg(hdst + 1, hp[1]);
-            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n));
-#pragma unroll
-            for (int v = 0; v < 4; ++v)
-                __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
-            if (T.c_all) {
-                float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
+                for (int v = 0; v < 16; ++v) {
+                    const float ig = sigmoid_approx(zi[v] + bi[v]);
+                    const float fg = sigmoid_approx(zf[v] + bf[v]);
+                    const float og = sigmoid_approx(zo[v] + bo[v]);
+                    const float gh = tanh_approx(zg[v] + bg[v]);
+                    const float cn = fmaf(fg, cp[v], ig * gh);
+                    cv[v] = cn;
+                    hv[v] = og * tanh_approx(cn);
+                }
+                uint4 hp[2];
+                hp[0] = make_uint4(pack_bf16x2(hv[0], hv[1]), pack_bf16x2(hv[2], hv[3]),
+                                   pack_bf16x2(hv[4], hv[5]), pack_bf16x2(hv[6], hv[7]));
+                hp[1] = make_uint4(pack_bf16x2(hv[8], hv[9]), pack_bf16x2(hv[10], hv[11]),
+                                   pack_bf16x2(hv[12], hv[13]), pack_bf16x2(hv[14], hv[15]));
+                const long long hi = h_all_index(P, c, tl.axis, b, n);
+                uint4* hdst = reinterpret_cast<uint4*>(h_all + hi);
+                __stcg(hdst + 0, hp[0]);
+                __stcg(hdst + 1, hp[1]);
+                float4* cdst =
+                    reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n));
 #pragma unroll
                 for (int v = 0; v < 4; ++v)
-                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
-            }
-            if (top) {
-                uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n));
-                d[0] = hp[0];
-                d[1] = hp[1];
-            }
-            if (last) {
-                const long long ni = hn_index(P, c, tl.axis, b, n);
-                uint4* d = reinterpret_cast<uint4*>(h_n + ni);
-                d[0] = hp[0];
-                d[1] = hp[1];
-                float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
+                    __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
+                if (T.c_all) {
+                    float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
 #pragma unroll
-                for (int v = 0; v < 4; ++v)
-                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+                    for (int v = 0; v < 4; ++v)
+                        d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+                }
+                if (top) {
+                    uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n));
+                    d[0] = hp[0];
+                    d[1] = hp[1];
+                }
+                if (last) {
+                    const long long ni = hn_index(P, c, tl.axis, b, n);
+                    uint4* d = reinterpret_cast<uint4*>(h_n + ni);
+                    d[0] = hp[0];
+                    d[1] = hp[1];
+                    float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
+#pragma unroll
+                    for (int v = 0; v < 4; ++v)
+                        d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+                }
             }
-            }  // valid
         }
-        // publish this tile's share of the (cell, m-block) readiness counter
+        // publish this CTA's share of the (cell, m-block) readiness counter
         __threadfence();
         named_bar_sync(1, 128);
         if (warp == 2 && lane == 0)
@@ -256,30 +316,33 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     }
 }
 
+template <int CG>
 __global__ void __launch_bounds__(THREADS, 1)
 wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
                       const __grid_constant__ Maps M) {
+    using C = KCfg<CG>;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     uint8_t* smem = smem_raw + pad;
     uint8_t* sA = smem;
-    uint8_t* sB = smem + STAGES * A_BYTES;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * STAGE_BYTES);
+    uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + C::STAGES * C::STAGE_BYTES);
     uint64_t* full = bars;
-    uint64_t* empty = bars + STAGES;
-    uint64_t* tfull = bars + 2 * STAGES;
+    uint64_t* empty = bars + C::STAGES;
+    uint64_t* tfull = bars + 2 * C::STAGES;
     uint64_t* tempty = tfull + 2;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
     if (threadIdx.x == 0) {
-        for (int s = 0; s < STAGES; ++s) {
+        for (int s = 0; s < C::STAGES; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], 1);
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull[a], 1);
-            mbar_init(&tempty[a], 4);
+            mbar_init(&tempty[a], 4 * CG);
         }
         fence_mbarrier_init();
         tma_prefetch_desc(&M.x);
@@ -288,25 +351,27 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         tma_prefetch_desc(&M.W);
         tma_prefetch_desc(&M.U);
     }
-    if (warp == 1) tmem_alloc(tmem_slot, TMEM_COLS);
+    if (warp == 1) tmem_alloc_cg<CG>(tmem_slot, TMEM_COLS);
     tc_fence_before();
     __syncthreads();
+    if constexpr (CG == 2) cluster_sync();
     tc_fence_after();
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == 0) {
-        if (lane == 0) run_producer(P, T, M, sA, sB, full, empty);
+        if (lane == 0) run_producer<CG>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
-        if (lane == 0) run_mma(P, tmem_base, sA, sB, full, empty, tfull, tempty);
+        if (lane == 0 && rank == 0) run_mma<CG>(P, tmem_base, sA, sB, full, empty, tfull, tempty);
     } else {
-        run_epilogue(P, T, tmem_base, tfull, tempty);
+        run_epilogue<CG>(P, T, tmem_base, tfull, tempty, rank);
     }
 
     tc_fence_before();
     __syncthreads();
+    if constexpr (CG == 2) cluster_sync();
     if (warp == 1) {
         tc_fence_after();
-        tmem_dealloc(tmem_base, TMEM_COLS);
+        tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
     }
 }
 
@@ -336,7 +401,7 @@ bool encode_act(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, long
                 int B, std::string* err) {
     const cuuint64_t dims[3] = {(cuuint64_t)H, (cuuint64_t)rows, (cuuint64_t)B};
     const cuuint64_t strides[2] = {(cuuint64_t)H * 2, (cuuint64_t)rows * H * 2};
-    const cuuint32_t box[3] = {(cuuint32_t)BK, 1, (cuuint32_t)BM};
+    const cuuint32_t box[3] = {(cuuint32_t)BK, 1, (cuuint32_t)ROWS};
     const cuuint32_t es[3] = {1, 1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides,
                      box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -348,14 +413,14 @@ bool encode_act(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, long
     return true;
 }
 
-// Weight view (n, k, gate, slice) with a (64, 64, 4, 1) box, 128-byte swizzle: one box is the
-// [i | f | o | ĝ] x 64-unit N-tile of one 64-row K-chunk.
+// Weight view (n, k, gate, slice) with a (64, 64, gates, 1) box, 128-byte swizzle: the box is
+// the [i | f | o | ĝ] (CG 1) or [i | f] / [o | ĝ] (CG 2) x 64-unit slab of one 64-row K chunk.
 bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int krows, int slices,
-               std::string* err) {
+               int gates, std::string* err) {
     const cuuint64_t dims[4] = {(cuuint64_t)H, (cuuint64_t)krows, 4, (cuuint64_t)slices};
     const cuuint64_t strides[3] = {(cuuint64_t)H * 2, (cuuint64_t)krows * H * 2,
                                    (cuuint64_t)4 * krows * H * 2};
-    const cuuint32_t box[4] = {(cuuint32_t)BNU, (cuuint32_t)BK, 4, 1};
+    const cuuint32_t box[4] = {(cuuint32_t)BNU, (cuuint32_t)BK, (cuuint32_t)gates, 1};
     const cuuint32_t es[4] = {1, 1, 1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides,
                      box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -367,10 +432,9 @@ bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int k
     return true;
 }
 
-}  // namespace
-
-cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
-                                  std::string* err) {
+template <int CG>
+cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+    using C = KCfg<CG>;
     EncodeTiledFn enc = get_encode_fn(err);
     if (!enc) return cudaErrorNotSupported;
     Maps M;
@@ -380,34 +444,63 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
                     p.kind == KIND_GRID ? p.L1 : p.L0, p.B, err))
         return cudaErrorInvalidValue;
     if (!encode_act(enc, &M.h, t.h_all, p.H, h_rows(p), p.B, err)) return cudaErrorInvalidValue;
-    if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, err)) return cudaErrorInvalidValue;
-    if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, err)) return cudaErrorInvalidValue;
+    if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, err)) return cudaErrorInvalidValue;
+    if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, err))
+        return cudaErrorInvalidValue;
 
     int dev = 0, nsm = 0;
     cudaError_t e = cudaGetDevice(&dev);
     if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(wavefront_bf16_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 SMEM_BYTES);
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) {
         if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
         return e;
     }
-    long long grid = nsm;
-    if (grid > p.ntiles) grid = p.ntiles;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)grid);
     cfg.blockDim = dim3(THREADS);
-    cfg.dynamicSmemBytes = SMEM_BYTES;
+    cfg.dynamicSmemBytes = C::SMEM_BYTES;
     cfg.stream = s;
     cudaLaunchAttribute attr[1];
-    attr[0].id = cudaLaunchAttributeCooperative;
-    attr[0].val.cooperative = 1;
+    long long grid;
+    if constexpr (CG == 1) {
+        grid = nsm;
+        if (grid > p.ntiles) grid = p.ntiles;
+        attr[0].id = cudaLaunchAttributeCooperative;  // all CTAs co-resident (spin-wait safety)
+        attr[0].val.cooperative = 1;
+    } else {
+        // Cluster launch: every cluster must be co-resident; size the grid by the number of
+        // clusters the device can hold at once (one CTA per SM, so <= nsm / 2).
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = 2;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.gridDim = dim3((unsigned)(nsm & ~1));
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        int nclusters = 0;
+        e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG>, &cfg);
+        if (e != cudaSuccess || nclusters < 1) {
+            if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
+            return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
+        }
+        grid = 2ll * nclusters;
+        if (grid > 2 * p.ntiles) grid = 2 * p.ntiles;
+    }
+    cfg.gridDim = dim3((unsigned)grid);
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel, p, t, M);
+    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG>, p, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
+}
+
+}  // namespace
+
+cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
+                                  std::string* err) {
+    return p.BM == 2 * ROWS ? launch_cg<2>(p, t, s, err) : launch_cg<1>(p, t, s, err);
 }
 
 }  // namespace ft
