@@ -59,8 +59,16 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
     p->BM = dt == FT_BF16 ? (B > ft::BF16_BM ? 2 * ft::BF16_BM : ft::BF16_BM) : ft::F32_BM;
     p->flag_mult = dt == FT_BF16 ? p->BM / ft::BF16_BM : 1;
     {
-        const char* env = getenv("FT_L2_RESIDENT_LAYERS");
-        p->resident_layers = env ? atoi(env) : 0;
+        // a5 weight residency: when every layer's weights fit in about half of the 126 MB L2
+        // they are kept there across time steps (EVICT_LAST); otherwise they stream (EVICT_FIRST)
+        // — a 256 MiB weight set cannot be resident, each diagonal re-reads it.
+        const double wbytes = (double)D * p->naxes * 4.0 * H * ((double)H + (kind == ft::KIND_SEQ ? H : 2.0 * H)) *
+                              (dt == FT_BF16 ? 2 : 4);
+        p->resident_layers = wbytes <= 64.0 * 1024 * 1024 ? D : 0;
+        const char* env = getenv("FT_L2_RESIDENT_LAYERS");  // tuning override
+        if (env) p->resident_layers = atoi(env);
+        const char* dbg = getenv("FT_DEBUG");  // timing experiments only
+        p->debug = dbg ? atoi(dbg) : 0;
     }
     p->BNU = dt == FT_BF16 ? ft::BF16_BNU : ft::F32_BNU;
     p->MB = (B + p->BM - 1) / p->BM;
@@ -94,9 +102,12 @@ WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
     w.hall_off = w.ring_off + w.ring_bytes;
-    w.hall_bytes = h_all_provided
-                       ? 0
-                       : round_up((size_t)p.B * ft::h_rows(p) * p.H * elem_size(dt), 256);
+    if (dt == FT_BF16)  // the blocked SSA activation buffer (always; the caller's h_all is a copy)
+        w.hall_bytes = round_up((size_t)ft::hb_rows_total(p) * 64 * 2, 256);
+    else
+        w.hall_bytes = h_all_provided
+                           ? 0
+                           : round_up((size_t)p.B * ft::h_rows(p) * p.H * elem_size(dt), 256);
     w.total = w.hall_off + w.hall_bytes;
     return w;
 }
@@ -128,7 +139,10 @@ ft_status run(const ft::Problem& p, ft_dtype dt, ft::Tensors t, void* workspace,
     uint8_t* ws = static_cast<uint8_t*>(workspace);
     t.flags = reinterpret_cast<int*>(ws + w.flags_off);
     t.c_ring = reinterpret_cast<float*>(ws + w.ring_off);
-    if (!t.h_all) t.h_all = ws + w.hall_off;
+    if (dt == FT_BF16)
+        t.hb = ws + w.hall_off;
+    else if (!t.h_all)
+        t.h_all = ws + w.hall_off;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     cudaError_t e = cudaMemsetAsync(t.flags, 0, w.flags_bytes, s);  // BK0: reset readiness flags
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("flag reset: ") + cudaGetErrorString(e));

@@ -34,6 +34,8 @@ struct Problem {
     int MB, NT;          // m-blocks = ceil(B/BM), n-tiles per axis = ceil(H/BNU)
     int flag_mult;       // counter increments per tile (CTAs per tile: 2 for a tcgen05 CTA pair)
     int resident_layers; // bf16: layers whose weights are kept in L2 (evict_last); others stream
+    int debug;           // timing experiments only (env FT_DEBUG; results invalid when != 0):
+                         // bit 0 skip dependency waits, bit 1 skip the epilogue math/stores
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT
     int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)
@@ -142,18 +144,19 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
 // Producer cells of (d, i, j) — the dependence vectors of Table 4 (L307–L317):
 // KIND_SEQ: e_depth → (d-1, t), s_d·e_time → (d, t - s_d) (strided access, L331).
 // KIND_GRID: e_depth, e_x, e_y → (d-1,i,j), (d,i-1,j), (d,i,j-1).
-// Returns the number of producers written to out[] (as linear cell indices).
+// Fixed slots (out[k] = linear cell index, or -1 when that producer is outside the domain), so
+// callers keep them in registers.  Returns the number of valid producers.
 FT_HD int producers(const Problem& p, const Cell& c, long long out[3]) {
-    int n = 0;
-    if (c.d > 0) out[n++] = cell_lin(p, c.d - 1, c.i, c.j);
+    out[0] = c.d > 0 ? cell_lin(p, c.d - 1, c.i, c.j) : -1;
     if (p.kind == KIND_SEQ) {
         const int s = p.dil[c.d];
-        if (c.i >= s) out[n++] = cell_lin(p, c.d, c.i - s, 0);
+        out[1] = c.i >= s ? cell_lin(p, c.d, c.i - s, 0) : -1;
+        out[2] = -1;
     } else {
-        if (c.i > 0) out[n++] = cell_lin(p, c.d, c.i - 1, c.j);
-        if (c.j > 0) out[n++] = cell_lin(p, c.d, c.i, c.j - 1);
+        out[1] = c.i > 0 ? cell_lin(p, c.d, c.i - 1, c.j) : -1;
+        out[2] = c.j > 0 ? cell_lin(p, c.d, c.i, c.j - 1) : -1;
     }
-    return n;
+    return (out[0] >= 0) + (out[1] >= 0) + (out[2] >= 0);
 }
 
 // ------------------------------------------------------------------------------------------
@@ -162,7 +165,7 @@ FT_HD int producers(const Problem& p, const Cell& c, long long out[3]) {
 // batch-outermost buffers.  An activation "row" is the middle coordinate of the
 // (hidden, rows, batch) view of a buffer: x/ys: position; h_all: (d, t) or (d, i, j, axis).
 // ------------------------------------------------------------------------------------------
-enum Src : int { SRC_X = 0, SRC_YS = 1, SRC_H = 2 };
+enum Src : int { SRC_X = 0, SRC_YS = 1, SRC_H = 2, SRC_NONE = 3 };
 enum WSel : int { W_IN = 0, W_REC = 1 };
 
 struct Segment {
@@ -183,28 +186,39 @@ FT_HD int h_row(const Problem& p, int d, int i, int j, int a) {
 // K rows of one U slice: H (seq) or 2H (grid, acting on s = [h^x; h^y]).
 FT_HD int u_krows(const Problem& p) { return p.kind == KIND_SEQ ? p.H : 2 * p.H; }
 
-// The A-operand segments of one tile (the vertical merge x@w + h@u of L609 as one K loop).
-// A segment whose producer is outside the domain (t < s, i = 0, j = 0) is the zero initial
-// state (scanl s0 = 0, L159/L605) and is skipped: that is the paper's boundary region split
-// (region_0..3, L243/L256).
+// The A-operand segments of one tile (the vertical merge x@w + h@u of L609 as one K loop), in
+// fixed slots: 0 = layer input, 1 = recurrent state (seq) / h^x_{i-1,j} (grid), 2 = h^y_{i,j-1}
+// (grid).  A segment whose producer is outside the domain (t < s, i = 0, j = 0) is the zero
+// initial state (scanl s0 = 0, L159/L605) and is marked invalid (skipped): that is the paper's
+// boundary region split (region_0..3, L243/L256).  Returns the number of valid segments.
 FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
     const Cell& c = tl.cell;
-    int n = 0;
     if (p.kind == KIND_SEQ) {
-        seg[n++] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0}
-                              : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0};
+        seg[0] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0}
+                            : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0};
         const int s = p.dil[c.d];
-        if (c.i >= s) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i - s, 0, 0), W_REC, c.d, 0};
-        return n;
+        seg[1] = Segment{c.i >= s ? SRC_H : SRC_NONE, c.i >= s ? h_row(p, c.d, c.i - s, 0, 0) : 0,
+                         W_REC, c.d, 0};
+        seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0};
+    } else {
+        const int a = tl.axis, sl = c.d * 2 + a;
+        if (c.d == 0)
+            seg[0] = Segment{a == 0 ? SRC_X : SRC_YS, a == 0 ? c.i : c.j, W_IN, sl, 0};
+        else
+            seg[0] = Segment{SRC_H, h_row(p, c.d - 1, c.i, c.j, a), W_IN, sl, 0};
+        seg[1] = Segment{c.i > 0 ? SRC_H : SRC_NONE, c.i > 0 ? h_row(p, c.d, c.i - 1, c.j, 0) : 0,
+                         W_REC, sl, 0};
+        seg[2] = Segment{c.j > 0 ? SRC_H : SRC_NONE, c.j > 0 ? h_row(p, c.d, c.i, c.j - 1, 1) : 0,
+                         W_REC, sl, p.H};
     }
-    const int a = tl.axis, sl = c.d * 2 + a;
-    if (c.d == 0)
-        seg[n++] = Segment{a == 0 ? SRC_X : SRC_YS, a == 0 ? c.i : c.j, W_IN, sl, 0};
-    else
-        seg[n++] = Segment{SRC_H, h_row(p, c.d - 1, c.i, c.j, a), W_IN, sl, 0};
-    if (c.i > 0) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i - 1, c.j, 0), W_REC, sl, 0};
-    if (c.j > 0) seg[n++] = Segment{SRC_H, h_row(p, c.d, c.i, c.j - 1, 1), W_REC, sl, p.H};
-    return n;
+    return 1 + (seg[1].src != SRC_NONE) + (seg[2].src != SRC_NONE);
+}
+
+// Index of the next valid segment after slot `si` (3 when none is left).
+FT_HD int next_segment(const Segment seg[3], int si) {
+    if (si < 1 && seg[1].src != SRC_NONE) return 1;
+    if (si < 2 && seg[2].src != SRC_NONE) return 2;
+    return 3;
 }
 
 // rows per batch row of each activation source
@@ -249,6 +263,17 @@ FT_HD long long c_producer(const Problem& p, const TileId& tl, int* pi, int* pj)
     *pi = c.i;
     *pj = c.j - 1;
     return cell_lin(p, c.d, c.i, c.j - 1);
+}
+
+// bf16 path: the SSA activations live in a blocked, batch-contiguous layout
+//   hb[row][kc][Bp][64]   (row = h_row(), kc = unit / 64, Bp = MB * BM batch rows incl. padding)
+// so that the A operand of one tile K-chunk (128 batch rows x 64 units) is one contiguous 16 KiB
+// block: a 2-D TMA box with no large strides, and the epilogue's h stores are coalesced.
+FT_HD long long hb_rows_total(const Problem& p) {
+    return (long long)h_rows(p) * (p.H / 64) * ((long long)p.MB * p.BM);
+}
+FT_HD long long hb_row(const Problem& p, int row, int kc, int b) {
+    return ((long long)row * (p.H / 64) + kc) * ((long long)p.MB * p.BM) + b;
 }
 
 // Output element indices (batch row b, unit n).

@@ -19,7 +19,8 @@ struct Tensors {
     void* y = nullptr;
     void* h_n = nullptr;
     float* c_n = nullptr;
-    void* h_all = nullptr;   // never NULL at launch (workspace stand-in if the caller passed NULL)
+    void* h_all = nullptr;   // f32 path: never NULL at launch (workspace stand-in); bf16: optional
+    void* hb = nullptr;      // bf16 path: blocked SSA activations [h_rows][H/64][Bp][64] (workspace)
     float* c_all = nullptr;  // optional
     float* c_ring = nullptr; // workspace: fp32 cell-state ring
     int* flags = nullptr;    // workspace: readiness counters [ncells][MB]

@@ -19,19 +19,19 @@
 //           issues M256 N256 K16 MMAs reading both CTAs' shared memory, so each weight tile is
 //           fetched once per cell for the whole 256-row batch and per-CTA weight traffic halves.
 //
-// Warp roles (192 threads per CTA):
+// Warp roles (320 threads per CTA):
 //   warp 0      TMA producer: waits the tile's producer cells (readiness counters), then streams
 //               64-deep K-chunks of A and B into a STAGES-deep shared-memory ring (mbarriers).
 //   warp 1      MMA issuer (leader CTA): one thread issues tcgen05.mma into a double-buffered
 //               TMEM accumulator (2 x 256 fp32 columns) so tile n+1's MMAs overlap tile n's
 //               epilogue.
-//   warps 2-5   epilogue: tcgen05.ld → +b, σ/σ/σ/tanh, c' = f·c + i·ĝ, h' = o·tanh(c') in fp32
+//   warps 2-9   epilogue (2 warps per TMEM lane quadrant, 32 units each): tcgen05.ld → +b, σ/σ/σ/tanh, c' = f·c + i·ĝ, h' = o·tanh(c') in fp32
 //               registers; h' → bf16 → h_all (the SSA buffer node, L217) and y / h_n; c' → fp32
 //               cell-state ring (+ c_all / c_n); then release the tile's share of the
 //               (cell, m-block) readiness counter.
 //
 // Cross-CTA ordering (generic-proxy stores → another SM's async-proxy TMA loads):
-//   writer: st.global …; fence.acq_rel.gpu (every thread); bar.sync; red.release.gpu
+//   writer: st.global …; bar.sync (epilogue warps); one thread fence.acq_rel.gpu + red.release.gpu
 //   reader: ld.acquire.gpu (bounded spin); fence.proxy.async.global; cp.async.bulk.tensor
 // L2 policy: streamed weights EVICT_FIRST (they are re-read only one diagonal later, after the
 // whole 256 MiB weight set went through L2), weights of the first `resident_layers` layers
@@ -47,6 +47,36 @@
 #include "ft_sm100.cuh"
 
 namespace ft {
+
+#ifdef FT_TRACE
+// Development-only role timing (built into libft_trace.so by tools/trace_build.sh, never into
+// libft.so): per CTA, cycles spent in each wait / work phase.
+enum TraceSlot {
+    TR_P_FLAG = 0, TR_P_EMPTY, TR_M_FULL, TR_M_TEMPTY, TR_E_TFULL, TR_E_WORK, TR_E_CFLAG, TR_TOTAL,
+    TR_TILES, TR_SLOTS = 16
+};
+__device__ unsigned long long g_trace[1024 * TR_SLOTS];
+// register accumulators, flushed once per role (keeps the instrumented loops lean)
+#define FT_TR_ROLE unsigned long long _acc[TR_SLOTS] = {0}
+#define FT_TR_DECL long long _tr0 = 0
+#define FT_TR_BEGIN() (_tr0 = clock64())
+#define FT_TR_END(slot) (_acc[(slot)] += (unsigned long long)(clock64() - _tr0))
+#define FT_TR_ADD(slot, v) (_acc[(slot)] += (unsigned long long)(v))
+#define FT_TR_FLUSH(cond)                                                          \
+    do {                                                                           \
+        if (cond)                                                                  \
+            for (int _k = 0; _k < TR_SLOTS; ++_k)                                  \
+                if (_acc[_k]) g_trace[blockIdx.x * TR_SLOTS + _k] += _acc[_k];     \
+    } while (0)
+#else
+#define FT_TR_ROLE
+#define FT_TR_DECL
+#define FT_TR_BEGIN() ((void)0)
+#define FT_TR_END(slot) ((void)0)
+#define FT_TR_ADD(slot, v) ((void)0)
+#define FT_TR_FLUSH(cond) ((void)0)
+#endif
+
 namespace {
 
 using namespace sm100;
@@ -56,7 +86,7 @@ constexpr int BNU = BF16_BNU;  // 64 hidden units per tile
 constexpr int BN = 4 * BNU;    // 256 = UMMA N (i | f | o | ĝ)
 constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16
 constexpr int UK = 16;         // UMMA K for kind::f16
-constexpr int THREADS = 192;
+constexpr int THREADS = 320;  // warp 0 TMA, warp 1 MMA, warps 2-9 epilogue
 constexpr int TMEM_COLS = 2 * BN;  // double-buffered accumulator
 
 template <int CG>
@@ -65,7 +95,10 @@ struct KCfg {
     static constexpr int A_BYTES = ROWS * BK * 2;              // 16 KiB
     static constexpr int B_BYTES = GATES * BNU * BK * 2;       // 32 KiB (CG 1) / 16 KiB (CG 2)
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-    static constexpr int STAGES = CG == 1 ? 4 : 6;
+#ifndef FT_STAGES2
+#define FT_STAGES2 6
+#endif
+    static constexpr int STAGES = CG == 1 ? 4 : FT_STAGES2;
     static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024;
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
 };
@@ -79,11 +112,42 @@ __device__ __forceinline__ int weight_layer(const Problem& P, int slice) {
 }
 
 // ------------------------------------------------------------------------------ producer
+// The weight (B) half of a stage does not depend on any other cell, only the activation (A) half
+// does.  So for each tile the producer first claims up to STAGES ring slots and starts their
+// weight loads (the HBM stream), THEN waits for the producer cells' readiness counters, then
+// issues the activation loads of those slots: the weight latency hides behind the dependency wait.
+// The loop is kept lean (no division, no local-memory arrays, precomputed shared addresses): one
+// thread must issue a 32–48 KiB stage every ~512 tensor cycles.
+__device__ __forceinline__ Segment pick(const Segment (&seg)[3], int i) {
+    Segment r;  // field-wise selects keep the three segments in registers
+    r.src = i == 0 ? seg[0].src : (i == 1 ? seg[1].src : seg[2].src);
+    r.row = i == 0 ? seg[0].row : (i == 1 ? seg[1].row : seg[2].row);
+    r.wsel = i == 0 ? seg[0].wsel : (i == 1 ? seg[1].wsel : seg[2].wsel);
+    r.slice = i == 0 ? seg[0].slice : (i == 1 ? seg[1].slice : seg[2].slice);
+    r.krow0 = i == 0 ? seg[0].krow0 : (i == 1 ? seg[1].krow0 : seg[2].krow0);
+    return r;
+}
+
+// A operand K-chunk kc of segment sg for batch rows arow0 .. arow0+127: layer-0 inputs from the
+// caller's x / ys (3-D strided view), SSA activations from the blocked hb buffer (2-D, contiguous).
+template <int CG>
+__device__ __forceinline__ void load_a(const Problem& P, const Maps& M, uint32_t dst, uint32_t bar,
+                                       const Segment& sg, int kc, int arow0, bool fixed, uint64_t pol) {
+    if (fixed || sg.src != SRC_H) {
+        const CUtensorMap* am = (fixed || sg.src == SRC_X) ? &M.x : &M.ys;
+        tma_load_3d_hint_addr<CG>(dst, am, bar, fixed ? 0 : kc * BK, fixed ? 0 : sg.row, arow0, pol);
+    } else {
+        tma_load_2d_hint_addr<CG>(dst, &M.h, bar, 0, (int)hb_row(P, sg.row, kc, arow0), pol);
+    }
+}
+
 template <int CG>
 __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
                                              uint8_t* sA, uint8_t* sB, uint64_t* full,
                                              uint64_t* empty, uint32_t rank) {
     using C = KCfg<CG>;
+    const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
+    const uint32_t full0 = (CG == 2) ? mapa_shared(smem_u32(full), 0) : smem_u32(full);
     int stage = 0;
     uint32_t phase = 0;
     Cursor cur = cursor_begin();
@@ -92,37 +156,70 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const uint64_t pol_stream = policy_evict_first();
     const uint64_t pol_keep = policy_evict_last();
     const uint64_t pol_act = policy_evict_normal();
+    const bool skipA = P.debug & 8, skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
+    const uint32_t tx = CG * ((skipA ? 0 : C::A_BYTES) + (skipB ? 0 : C::B_BYTES));
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
-        long long prod[3];
-        const int np = producers(P, tl.cell, prod);
-        for (int q = 0; q < np; ++q) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
-        fence_proxy_async_global();
         Segment seg[3];
         const int ns = segments(P, tl, seg);
+        const int nchunks = ns * kchunks;
+        const int npre = nchunks < C::STAGES ? nchunks : C::STAGES;
         const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
-        for (int s = 0; s < ns; ++s) {
-            const CUtensorMap* am = seg[s].src == SRC_X ? &M.x : (seg[s].src == SRC_YS ? &M.ys : &M.h);
-            const CUtensorMap* bm = seg[s].wsel == W_IN ? &M.W : &M.U;
-            const uint64_t wpol = weight_layer(P, seg[s].slice) < P.resident_layers ? pol_keep : pol_stream;
-            for (int kc = 0; kc < kchunks; ++kc) {
-                mbar_wait(&empty[stage], phase ^ 1);
-                uint32_t bar = smem_u32(&full[stage]);
-                if constexpr (CG == 2) bar = mapa_shared(bar, 0);  // the leader's barrier
-                if (rank == 0) mbar_arrive_expect_tx(&full[stage], CG * C::STAGE_BYTES);
-                tma_load_3d_hint<CG>(sA + stage * C::A_BYTES, am, bar, kc * BK, seg[s].row, arow0,
-                                     pol_act);
-                tma_load_4d_hint<CG>(sB + stage * C::B_BYTES, bm, bar, tl.n * BNU,
-                                     seg[s].krow0 + kc * BK, (int)rank * C::GATES, seg[s].slice,
-                                     wpol);
-                if (++stage == C::STAGES) {
-                    stage = 0;
-                    phase ^= 1;
+        const int bn = fixed ? 0 : tl.n * BNU;
+        const int bg = (int)rank * C::GATES;
+        FT_TR_DECL;
+        int first_stage = stage;
+        int si = 0, kc = 0;
+        for (int c = 0; c < nchunks; ++c) {
+            const Segment sg = pick(seg, si);
+            FT_TR_BEGIN();
+            mbar_wait(&empty[stage], phase ^ 1);
+            FT_TR_END(TR_P_EMPTY);
+            const uint32_t bar = full0 + 8u * (uint32_t)stage;
+            if (rank == 0) mbar_arrive_expect_tx(&full[stage], tx);
+            if (!skipB) {
+                const CUtensorMap* bm = sg.wsel == W_IN ? &M.W : &M.U;
+                const uint64_t wpol = weight_layer(P, sg.slice) < P.resident_layers ? pol_keep : pol_stream;
+                tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
+                                          fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
+            }
+            if (c >= npre) {
+                if (!skipA) load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
+            } else if (c + 1 == npre) {
+                // dependencies (Table 4 vectors) of this tile, then the deferred A loads
+                long long prod[3];
+                const int np = producers(P, tl.cell, prod);
+                FT_TR_BEGIN();
+                if (!(P.debug & 1)) {
+#pragma unroll
+                    for (int q = 0; q < 3; ++q)
+                        if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
                 }
+                (void)np;
+                FT_TR_END(TR_P_FLAG);
+                FT_TR_ADD(TR_TILES, 1);
+                fence_proxy_async_global();
+                if (!skipA) {
+                    int ps = first_stage, psi = 0, pkc = 0;
+                    for (int cc = 0; cc < npre; ++cc) {
+                        const Segment sa = pick(seg, psi);
+                        load_a<CG>(P, M, sA0 + (uint32_t)(ps * C::A_BYTES), full0 + 8u * (uint32_t)ps,
+                                   sa, pkc, arow0, fixed, pol_act);
+                        if (++ps == C::STAGES) ps = 0;
+                        if (++pkc == kchunks) { pkc = 0; psi = next_segment(seg, psi); }
+                    }
+                }
+            }
+            if (++kc == kchunks) { kc = 0; si = next_segment(seg, si); }
+            if (++stage == C::STAGES) {
+                stage = 0;
+                phase ^= 1;
             }
         }
     }
+    FT_TR_FLUSH(true);
 }
 
 // ------------------------------------------------------------------------------ MMA issuer
@@ -137,36 +234,63 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
     uint32_t acc_phase = 0;
     Cursor cur = cursor_begin();
     const int kchunks = P.H / BK;
+    // A: K-major, SW128: 128-B rows, 8-row groups 1024 B apart (SBO); K step = +32 B.
+    // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups 1024 B apart
+    //    (SBO); K step of 16 rows = +2048 B.  CG 2: each CTA holds half the gate atoms.
+    const uint64_t adesc0 = make_sdesc(smem_u32(sA), 16, 1024);
+    const uint64_t bdesc0 = make_sdesc(smem_u32(sB), 8192, 1024);
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
         Segment seg[3];
         const int nchunks = segments(P, tl, seg) * kchunks;
+        FT_TR_DECL;
+        FT_TR_BEGIN();
         mbar_wait(&tempty[acc], acc_phase ^ 1);
+        FT_TR_END(TR_M_TEMPTY);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
         for (int c = 0; c < nchunks; ++c) {
+            FT_TR_BEGIN();
             mbar_wait(&full[stage], phase);
+            FT_TR_END(TR_M_FULL);
             tc_fence_after();
-            // A: K-major, SW128: 128-B rows, 8-row groups 1024 B apart (SBO); K step = +32 B.
-            // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups 1024 B
-            //    apart (SBO); K step of 16 rows = +2048 B.  CG 2: each CTA holds half the atoms.
-            const uint64_t ad = make_sdesc(smem_u32(sA + stage * C::A_BYTES), 16, 1024);
-            const uint64_t bd = make_sdesc(smem_u32(sB + stage * C::B_BYTES), 8192, 1024);
+            if (P.debug & 4) {  // timing experiment: no MMA, hand the slot straight back
+                if constexpr (CG == 1) {
+                    mbar_arrive(&empty[stage]);
+                } else {
+                    mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 0));
+                    mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 1));
+                }
+            } else {
+            const uint64_t ad = adesc0 + (uint64_t)((stage * C::A_BYTES) >> 4);
+            const uint64_t bd = bdesc0 + (uint64_t)((stage * C::B_BYTES) >> 4);
 #pragma unroll
             for (int kk = 0; kk < BK / UK; ++kk)
                 umma_f16_cg<CG>(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
                                 bd + (uint64_t)((kk * UK * 128) >> 4), C::IDESC, (c | kk) != 0);
             umma_commit_cg<CG>(&empty[stage]);
+            }
             if (++stage == C::STAGES) {
                 stage = 0;
                 phase ^= 1;
             }
         }
-        umma_commit_cg<CG>(&tfull[acc]);
+        if (P.debug & 4) {
+            if constexpr (CG == 1) {
+                mbar_arrive(&tfull[acc]);
+            } else {
+                mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 0));
+                mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 1));
+            }
+        } else {
+            umma_commit_cg<CG>(&tfull[acc]);
+        }
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
+    FT_TR_FLUSH(true);
 }
 
 // ------------------------------------------------------------------------------ epilogue
@@ -187,12 +311,20 @@ __device__ __forceinline__ void load16(const float* src, float (&v)[16]) {
     }
 }
 
+// 8 epilogue warps: warp w reads TMEM lane quadrant w % 4 (rows) and unit half (w - 2) / 4
+// (32 of the tile's 64 units); one thread per batch row.
+constexpr int EPI_WARPS = 8;
+constexpr int EPI_THREADS = EPI_WARPS * 32;
+constexpr int EPI_UNITS = BNU / 2;  // units per thread
+
 template <int CG>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
                                              uint64_t* tfull, uint64_t* tempty, uint32_t rank) {
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int q = warp & 3;  // TMEM lane quadrant this warp may access
+    const int q = warp & 3;                 // TMEM lane quadrant this warp may access
+    const int half = (warp - 2) >> 2;       // which 32 units of the tile
     const int row = q * 32 + lane;
+    const bool leader_thread = (threadIdx.x == 64);
     int acc = 0;
     uint32_t acc_phase = 0;
     Cursor cur = cursor_begin();
@@ -201,23 +333,54 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     __nv_bfloat16* y = (__nv_bfloat16*)T.y;
     __nv_bfloat16* h_n = (__nv_bfloat16*)T.h_n;
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
         const Cell c = tl.cell;
         int ci = 0, cj = 0;
         const long long cprod = c_producer(P, tl, &ci, &cj);
-        if (cprod >= 0) wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
-        mbar_wait(&tfull[acc], acc_phase);
-        tc_fence_after();
-
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
+        const int n0 = tl.n * BNU + half * EPI_UNITS;
+        FT_TR_DECL;
+        // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
+        //     of the c-producer's counter, published to the other epilogue threads by bar.sync
+        FT_TR_BEGIN();
+        if (cprod >= 0 && leader_thread && !(P.debug & 1))
+            wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
+        named_bar_sync(1, EPI_THREADS);
+        if (leader_thread) FT_TR_END(TR_E_CFLAG);
+        float cp[EPI_UNITS];
+        if (cprod >= 0 && valid) {
+            const float4* src = reinterpret_cast<const float4*>(
+                T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n0));
+#pragma unroll
+            for (int v = 0; v < EPI_UNITS / 4; ++v) {
+                const float4 t4 = __ldcg(src + v);
+                cp[4 * v + 0] = t4.x;
+                cp[4 * v + 1] = t4.y;
+                cp[4 * v + 2] = t4.z;
+                cp[4 * v + 3] = t4.w;
+            }
+        } else {
+#pragma unroll
+            for (int v = 0; v < EPI_UNITS; ++v) cp[v] = 0.f;
+        }
+        FT_TR_BEGIN();
+        mbar_wait(&tfull[acc], acc_phase);
+        if (leader_thread) FT_TR_END(TR_E_TFULL);
+        FT_TR_BEGIN();
+        tc_fence_after();
+
         const int slice = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
         const float* bias = T.b + (long long)slice * 4 * P.H;
         const bool top = (c.d == P.D - 1), last = is_last_pos(P, c);
-        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16);
-#pragma unroll 1
-        for (int u0 = 0; u0 < BNU; u0 += 16) {
+        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
+                               (uint32_t)(half * EPI_UNITS);
+        uint4 hp[EPI_UNITS / 8];
+        float cv[EPI_UNITS];
+#pragma unroll
+        for (int u0 = 0; u0 < EPI_UNITS; u0 += 16) {
             __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
             float zi[16], zf[16], zo[16], zg[16];
             tmem_ld_32x32b_x16(tbase + 0 * BNU + u0, zi);
@@ -225,7 +388,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             tmem_ld_32x32b_x16(tbase + 2 * BNU + u0, zo);
             tmem_ld_32x32b_x16(tbase + 3 * BNU + u0, zg);
             tmem_wait_ld();
-            if (u0 + 16 == BNU) {  // accumulator buffer drained → hand it back to the MMA warp
+            if (u0 + 16 == EPI_UNITS) {  // accumulator drained → hand it back to the MMA warp
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) {
@@ -235,85 +398,83 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                         mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[acc]), 0));
                 }
             }
-            if (valid) {
-                const int n = tl.n * BNU + u0;
-                float cp[16];
-                if (cprod >= 0) {
-                    const float4* src = reinterpret_cast<const float4*>(
-                        T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n));
+            if (P.debug & 2) continue;
+            const int n = n0 + u0;
+            float bi[16], bf[16], bo[16], bg[16];
+            load16(bias + 0 * P.H + n, bi);
+            load16(bias + 1 * P.H + n, bf);
+            load16(bias + 2 * P.H + n, bo);
+            load16(bias + 3 * P.H + n, bg);
+            float hv[16];
 #pragma unroll
-                    for (int v = 0; v < 4; ++v) {
-                        const float4 t4 = __ldcg(src + v);
-                        cp[4 * v + 0] = t4.x;
-                        cp[4 * v + 1] = t4.y;
-                        cp[4 * v + 2] = t4.z;
-                        cp[4 * v + 3] = t4.w;
-                    }
-                } else {
+            for (int v = 0; v < 16; ++v) {
+                const float ig = sigmoid_approx(zi[v] + bi[v]);
+                const float fg = sigmoid_approx(zf[v] + bf[v]);
+                const float og = sigmoid_approx(zo[v] + bo[v]);
+                const float gh = tanh_approx(zg[v] + bg[v]);
+                const float cn = fmaf(fg, cp[u0 + v], ig * gh);
+                cv[u0 + v] = cn;
+                hv[v] = og * tanh_approx(cn);
+            }
 #pragma unroll
-                    for (int v = 0; v < 16; ++v) cp[v] = 0.f;
-                }
-                float bi[16], bf[16], bo[16], bg[16];
-                load16(bias + 0 * P.H + n, bi);
-                load16(bias + 1 * P.H + n, bf);
-                load16(bias + 2 * P.H + n, bo);
-                load16(bias + 3 * P.H + n, bg);
-                float hv[16], cv[16];
+            for (int w = 0; w < 2; ++w)
+                hp[u0 / 8 + w] = make_uint4(pack_bf16x2(hv[8 * w + 0], hv[8 * w + 1]),
+                                            pack_bf16x2(hv[8 * w + 2], hv[8 * w + 3]),
+                                            pack_bf16x2(hv[8 * w + 4], hv[8 * w + 5]),
+                                            pack_bf16x2(hv[8 * w + 6], hv[8 * w + 7]));
+        }
+        // (2) what downstream cells read: h (blocked SSA buffer hb) and c (ring) → publish
+        const long long hi = h_all_index(P, c, tl.axis, b, n0);
+        if (valid && !(P.debug & 2)) {
+            const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
+            uint4* hdst = reinterpret_cast<uint4*>(
+                (__nv_bfloat16*)T.hb + hb_row(P, row_h, n0 / 64, b) * 64 + (n0 % 64));
 #pragma unroll
-                for (int v = 0; v < 16; ++v) {
-                    const float ig = sigmoid_approx(zi[v] + bi[v]);
-                    const float fg = sigmoid_approx(zf[v] + bf[v]);
-                    const float og = sigmoid_approx(zo[v] + bo[v]);
-                    const float gh = tanh_approx(zg[v] + bg[v]);
-                    const float cn = fmaf(fg, cp[v], ig * gh);
-                    cv[v] = cn;
-                    hv[v] = og * tanh_approx(cn);
-                }
-                uint4 hp[2];
-                hp[0] = make_uint4(pack_bf16x2(hv[0], hv[1]), pack_bf16x2(hv[2], hv[3]),
-                                   pack_bf16x2(hv[4], hv[5]), pack_bf16x2(hv[6], hv[7]));
-                hp[1] = make_uint4(pack_bf16x2(hv[8], hv[9]), pack_bf16x2(hv[10], hv[11]),
-                                   pack_bf16x2(hv[12], hv[13]), pack_bf16x2(hv[14], hv[15]));
-                const long long hi = h_all_index(P, c, tl.axis, b, n);
-                uint4* hdst = reinterpret_cast<uint4*>(h_all + hi);
-                __stcg(hdst + 0, hp[0]);
-                __stcg(hdst + 1, hp[1]);
-                float4* cdst =
-                    reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n));
+            for (int w = 0; w < EPI_UNITS / 8; ++w) __stcg(hdst + w, hp[w]);
+            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n0));
 #pragma unroll
-                for (int v = 0; v < 4; ++v)
-                    __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
-                if (T.c_all) {
-                    float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
+            for (int v = 0; v < EPI_UNITS / 4; ++v)
+                __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
+        }
+        named_bar_sync(1, EPI_THREADS);
+        if (leader_thread) {
+            __threadfence();
+            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+            FT_TR_END(TR_E_WORK);
+        }
+        // (3) outputs nobody inside the nest reads
+        if (valid) {
+            if (h_all) {
+                uint4* d = reinterpret_cast<uint4*>(h_all + hi);
 #pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
-                }
-                if (top) {
-                    uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n));
-                    d[0] = hp[0];
-                    d[1] = hp[1];
-                }
-                if (last) {
-                    const long long ni = hn_index(P, c, tl.axis, b, n);
-                    uint4* d = reinterpret_cast<uint4*>(h_n + ni);
-                    d[0] = hp[0];
-                    d[1] = hp[1];
-                    float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
+                for (int w = 0; w < EPI_UNITS / 8; ++w) d[w] = hp[w];
+            }
+            if (T.c_all) {
+                float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
 #pragma unroll
-                    for (int v = 0; v < 4; ++v)
-                        d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
-                }
+                for (int v = 0; v < EPI_UNITS / 4; ++v)
+                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+            }
+            if (top) {
+                uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n0));
+#pragma unroll
+                for (int w = 0; w < EPI_UNITS / 8; ++w) d[w] = hp[w];
+            }
+            if (last) {
+                const long long ni = hn_index(P, c, tl.axis, b, n0);
+                uint4* d = reinterpret_cast<uint4*>(h_n + ni);
+#pragma unroll
+                for (int w = 0; w < EPI_UNITS / 8; ++w) d[w] = hp[w];
+                float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
+#pragma unroll
+                for (int v = 0; v < EPI_UNITS / 4; ++v)
+                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
             }
         }
-        // publish this CTA's share of the (cell, m-block) readiness counter
-        __threadfence();
-        named_bar_sync(1, 128);
-        if (warp == 2 && lane == 0)
-            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
+    FT_TR_FLUSH(leader_thread);
 }
 
 template <int CG>
@@ -335,6 +496,9 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
+    FT_TR_ROLE;
+    FT_TR_DECL;
+    FT_TR_BEGIN();
     if (threadIdx.x == 0) {
         for (int s = 0; s < C::STAGES; ++s) {
             mbar_init(&full[s], 1);
@@ -342,7 +506,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull[a], 1);
-            mbar_init(&tempty[a], 4 * CG);
+            mbar_init(&tempty[a], 8 * CG);
         }
         fence_mbarrier_init();
         tma_prefetch_desc(&M.x);
@@ -373,6 +537,8 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         tc_fence_after();
         tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
     }
+    if (threadIdx.x == 0) FT_TR_END(TR_TOTAL);
+    FT_TR_FLUSH(threadIdx.x == 0);
 }
 
 // ------------------------------------------------------------------------------ host side
@@ -413,6 +579,24 @@ bool encode_act(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, long
     return true;
 }
 
+// Blocked activation view (64 units, rows) with a (64, 128) box: one box = one contiguous 16 KiB
+// K-chunk of 128 batch rows.
+bool encode_blocked(EncodeTiledFn enc, CUtensorMap* m, const void* base, long long rows,
+                    std::string* err) {
+    const cuuint64_t dims[2] = {64, (cuuint64_t)rows};
+    const cuuint64_t strides[1] = {128};
+    const cuuint32_t box[2] = {(cuuint32_t)BK, (cuuint32_t)ROWS};
+    const cuuint32_t es[2] = {1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides,
+                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+        if (err) *err = "cuTensorMapEncodeTiled(blocked activation) failed: " + std::to_string((int)r);
+        return false;
+    }
+    return true;
+}
+
 // Weight view (n, k, gate, slice) with a (64, 64, gates, 1) box, 128-byte swizzle: the box is
 // the [i | f | o | ĝ] (CG 1) or [i | f] / [o | ĝ] (CG 2) x 64-unit slab of one 64-row K chunk.
 bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int krows, int slices,
@@ -443,7 +627,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     if (!encode_act(enc, &M.ys, p.kind == KIND_GRID ? t.ys : t.x, p.H,
                     p.kind == KIND_GRID ? p.L1 : p.L0, p.B, err))
         return cudaErrorInvalidValue;
-    if (!encode_act(enc, &M.h, t.h_all, p.H, h_rows(p), p.B, err)) return cudaErrorInvalidValue;
+    if (!encode_blocked(enc, &M.h, t.hb, hb_rows_total(p), err)) return cudaErrorInvalidValue;
     if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, err)) return cudaErrorInvalidValue;
     if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, err))
         return cudaErrorInvalidValue;
@@ -497,6 +681,20 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
 }
 
 }  // namespace
+
+#ifdef FT_TRACE
+extern "C" __attribute__((visibility("default"))) int ft_debug_trace(unsigned long long* host,
+                                                                     int n, int reset) {
+    if (n > 1024 * TR_SLOTS) n = 1024 * TR_SLOTS;
+    cudaDeviceSynchronize();
+    if (cudaMemcpyFromSymbol(host, g_trace, n * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    if (reset) {
+        static unsigned long long zeros[1024 * TR_SLOTS];
+        cudaMemcpyToSymbol(g_trace, zeros, sizeof(zeros));
+    }
+    return TR_SLOTS;
+}
+#endif
 
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
                                   std::string* err) {

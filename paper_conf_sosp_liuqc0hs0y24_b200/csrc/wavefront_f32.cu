@@ -48,8 +48,9 @@ wavefront_f32_kernel(const __grid_constant__ Problem P, const __grid_constant__ 
         // ---- wait for producer cells (Table 4 dependence vectors) ----------------------
         if (tid == 0) {
             long long prod[3];
-            const int np = producers(P, c, prod);
-            for (int q = 0; q < np; ++q) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
+            producers(P, c, prod);
+            for (int q = 0; q < 3; ++q)
+                if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
             __threadfence();
         }
         __syncthreads();
@@ -66,8 +67,9 @@ wavefront_f32_kernel(const __grid_constant__ Problem P, const __grid_constant__ 
             for (int r = 0; r < 4; ++r) acc[r][g] = bv;
         }
         Segment seg[3];
-        const int nseg = segments(P, tl, seg);
-        for (int s = 0; s < nseg; ++s) {
+        segments(P, tl, seg);
+        for (int s = 0; s < 3; ++s) {
+            if (seg[s].src == SRC_NONE) continue;
             const float* A = src_base(T, seg[s].src);
             const long long arows = src_rows(P, seg[s].src);
             const float* Wt = (const float*)(seg[s].wsel == W_IN ? T.W : T.U);

@@ -97,8 +97,11 @@ def test_workspace_sizes():
     B, T, H, D = 256, 100, 1024, 16
     with_h = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_BF16, True)
     without = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_BF16, False)
-    assert without - with_h >= B * D * T * H * 2  # the h_all SSA buffer lives in the workspace
-    assert with_h >= D * T * 2 * 4 + D * 2 * B * H * 4  # flags + 2-slot c ring
+    # bf16: the blocked SSA activation buffer always lives in the workspace (a caller h_all is a copy)
+    assert without == with_h >= B * D * T * H * 2 + D * T * 4 + D * 2 * B * H * 4
+    f_with = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_F32, True)
+    f_without = ft.ft_stacked_lstm_workspace_size(B, T, H, D, ft.FT_F32, False)
+    assert f_without - f_with >= B * D * T * H * 4  # fp32: h_all stand-in only when NULL
     assert ft.ft_dilated_rnn_workspace_size(B, T, H, D, [1] * D, ft.FT_BF16, True) == with_h
     big = ft.ft_dilated_rnn_workspace_size(B, T, H, D, [32] * D, ft.FT_BF16, True)
     assert big > with_h  # ring of 2·s slots per layer

@@ -16,7 +16,11 @@ def timeit(fn, reps=10, warm=3):
 
 res = {}
 for name in sys.argv[1:] or ["C2", "C3", "C4", "C5"]:
-    c = ftgen.CONFIGS[name]
+    if ":" in name:  # custom stacked spec  name:B,T,H,D
+        B_, T_, H_, D_ = (int(v) for v in name.split(":")[1].split(","))
+        c = dict(kind="stacked", batch=B_, seq=T_, hidden=H_, depth=D_)
+    else:
+        c = ftgen.CONFIGS[name]
     ws = ft.Workspace()
     if c["kind"] == "grid":
         g = ftgen.grid_inputs(c["batch"], c["len_x"], c["len_y"], c["hidden"], c["depth"], 1, "bf16")
