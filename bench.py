@@ -77,7 +77,7 @@ def load_traffic():
 class ClockSampler:
     FIELDS = ("timestamp,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap,utilization.gpu")
+              "clocks_event_reasons.sw_power_cap,utilization.gpu,power.draw")
 
     def __init__(self, index):
         self.index = index
@@ -107,12 +107,12 @@ class ClockSampler:
         with open(self.path) as f:
             for line in f:
                 parts = [x.strip() for x in line.split(",")]
-                if len(parts) < 8:
+                if len(parts) < 9:
                     continue
                 try:
                     rows.append(dict(sm=float(parts[1]), smax=float(parts[2]),
                                      hw=parts[3], hwt=parts[4], swt=parts[5], pc=parts[6],
-                                     util=float(parts[7])))
+                                     util=float(parts[7]), pw=float(parts[8])))
                 except ValueError:
                     continue
         os.unlink(self.path)
@@ -127,6 +127,7 @@ class ClockSampler:
                     reasons.add(name)
         return {"sm_mhz": statistics.median(r["sm"] for r in loaded),
                 "sm_max_mhz": max(r["smax"] for r in loaded), "reasons": sorted(reasons),
+                "power_w_median": statistics.median(r["pw"] for r in loaded),
                 "samples": len(loaded)}
 
 
@@ -233,12 +234,12 @@ def run_ours(args):
     outs = {"y": torch.empty((B, T, H), dtype=bf, device=dev),
             "h_n": torch.empty((B, D, H), dtype=bf, device=dev),
             "c_n": torch.empty((B, D, H), dtype=torch.float32, device=dev)}
-    gather_list = [torch.empty_like(outs["y"]) for _ in range(world)] if (args.gather and rank == 0) else None
+    from paper_conf_sosp_liuqc0hs0y24_b200.shard import gather_rows
 
     def step():
         ft.stacked_lstm(x, W, U, b, workspace=ws, out=outs)
-        if args.gather and world > 1:
-            dist.gather(outs["y"], gather_list, dst=0)
+        if args.gather and world > 1:  # the final output gather of y to rank 0 (NCCL / NVLink)
+            gather_rows(outs["y"], B * world, dst=0)
 
     stream = torch.cuda.current_stream()
     sampler = ClockSampler(local)

@@ -1,5 +1,5 @@
 """Quick device timing of the forward (development aid; bench.py is the contract)."""
-import sys, time, json
+import sys, time, json, os
 import numpy as np, torch
 sys.path.insert(0, ".")
 import ftgen
@@ -37,6 +37,6 @@ for name in sys.argv[1:] or ["C2", "C3", "C4", "C5"]:
             flops = sum(2*B*4*H*(H*T + H*max(0, T-s)) for s in dil)
         else:
             flops = 16 * H * H * T * D * B
-    med, mn = timeit(fn)
+    med, mn = timeit(fn, reps=int(os.environ.get("QT_REPS", "10")), warm=int(os.environ.get("QT_WARM", "3")))
     res[name] = dict(ms_median=med, ms_min=mn, tflops=flops / med / 1e9, seq_per_s=c["batch"] / med * 1e3)
     print(name, json.dumps(res[name]), flush=True)
