@@ -41,6 +41,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <string>
 
 #include "ft_internal.h"
@@ -698,6 +699,16 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_trace(unsigned lo
 
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
                                   std::string* err) {
+    // a5: weights resident in shared memory for the whole sequence when they fit
+    const char* env = getenv("FT_RESIDENT");  // "0" forces the streaming kernel (comparisons)
+    if (p.BM == ROWS && !(env && env[0] == '0')) {
+        int dev = 0, nsm = 0;
+        if (cudaGetDevice(&dev) == cudaSuccess &&
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess) {
+            const int bnu = resident_bnu(p, nsm);
+            if (bnu) return launch_wavefront_resident(p, t, s, bnu, err);
+        }
+    }
     return p.BM == 2 * ROWS ? launch_cg<2>(p, t, s, err) : launch_cg<1>(p, t, s, err);
 }
 

@@ -125,6 +125,18 @@ def test_bf16_small_and_ragged(B, T, H, D):
     _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"bf16 {B,T,H,D}")
 
 
+@pytest.mark.parametrize("mode", ["resident", "streaming"])
+@pytest.mark.parametrize("B,T,H,D", [(64, 9, 256, 8), (100, 5, 320, 3), (7, 6, 128, 4),
+                                     (32, 5, 256, 16)])  # last: 32-unit slabs (SW64 weights)
+def test_bf16_resident_vs_streaming(mode, B, T, H, D, monkeypatch):
+    """a5: the weight-resident kernel (weights in SMEM for the whole sequence, c in registers)
+    and the streaming kernel both match the oracle on shapes where the weights fit."""
+    monkeypatch.setenv("FT_RESIDENT", "1" if mode == "resident" else "0")
+    p = ftgen.stacked_inputs(B, T, H, D, 707 + H, "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"{mode} {B,T,H,D}")
+
+
 def test_bf16_C2_full():
     c = ftgen.CONFIGS["C2"]
     p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C2"), "bf16")
