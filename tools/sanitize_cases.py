@@ -1,0 +1,26 @@
+"""Small invocations of every kernel for compute-sanitizer (development aid)."""
+import sys, os
+import torch
+sys.path.insert(0, ".")
+import ftgen
+from paper_conf_sosp_liuqc0hs0y24_b200 import ft
+dev = "cuda"
+def run_seq(B, T, H, D, dt, dil=None, resident="1"):
+    os.environ["FT_RESIDENT"] = resident
+    p = ftgen.stacked_inputs(B, T, H, D, 1, "bf16" if dt == torch.bfloat16 else "f32")
+    a = [torch.from_numpy(p[k]).to(dev, dt) for k in ("x", "W", "U")] + [torch.from_numpy(p["b"]).to(dev)]
+    r = ft.stacked_lstm(*a, dilations=dil, want_all=True)
+    torch.cuda.synchronize()
+def run_grid(B, Lx, Ly, H, D, dt):
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, 1, "bf16" if dt == torch.bfloat16 else "f32")
+    a = [torch.from_numpy(g[k]).to(dev, dt) for k in ("x", "ys", "W", "U")] + [torch.from_numpy(g["b"]).to(dev)]
+    ft.grid_rnn(*a, want_all=True)
+    torch.cuda.synchronize()
+run_seq(4, 5, 64, 2, torch.float32)
+run_seq(5, 6, 128, 3, torch.bfloat16)                 # resident
+run_seq(5, 6, 128, 3, torch.bfloat16, resident="0")   # streaming, 1 CTA
+run_seq(130, 4, 128, 2, torch.bfloat16)               # streaming, CTA pair
+run_seq(20, 7, 128, 3, torch.bfloat16, dil=[1, 2, 3])
+run_grid(3, 3, 4, 64, 2, torch.bfloat16)
+run_grid(3, 3, 4, 16, 2, torch.float32)
+print("sanitize cases done")

@@ -34,7 +34,7 @@ __global__ void __launch_bounds__(128, 1) tma_loop(const __grid_constant__ CUten
     long long t0 = clock64();
     int s = 0;
     uint32_t phase = 0;
-    int c = blockIdx.x % ncoord;
+    int c = (int)(((long long)blockIdx.x * ncoord) / gridDim.x);
     for (int i = 0; i < iters; ++i) {
         const uint32_t bar = bar0 + 8 * s;
         if (i >= STAGES) {
@@ -52,7 +52,7 @@ __global__ void __launch_bounds__(128, 1) tma_loop(const __grid_constant__ CUten
                              ::"r"(dst), "l"((uint64_t)&map), "r"(bar), "r"(0), "r"(c), "r"(0), "l"(pol) : "memory");
             else if (RANK == 2)
                 asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];"
-                             ::"r"(dst), "l"((uint64_t)&map), "r"(bar), "r"(0), "r"(c * 8) : "memory");
+                             ::"r"(dst), "l"((uint64_t)&map), "r"(bar), "r"(0), "r"(c * 256) : "memory");
             else if (RANK == 3)
                 asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5}], [%2];"
                              ::"r"(dst), "l"((uint64_t)&map), "r"(bar), "r"(0), "r"(c), "r"(0) : "memory");
@@ -90,6 +90,10 @@ int main() {
     unsigned long long* out;
     CK(cudaMalloc(&out, 148 * sizeof(unsigned long long)));
     int nsm = 148;
+    void* big;
+    const size_t big_bytes = 2ull << 30;  // 2 GiB: no L2 reuse
+    CK(cudaMalloc(&big, big_bytes));
+    CK(cudaMemset(big, 1, big_bytes));
     struct Case { const char* name; int rank; cuuint64_t dims[4]; cuuint64_t strides[3]; cuuint32_t box[4]; CUtensorMapSwizzle sw; int ncoord; };
     std::vector<Case> cases = {
         // 2-D K-major operand tile: 64 bf16 (128 B) x 128 rows, rows 2 KB apart
@@ -104,6 +108,39 @@ int main() {
         {"4D 64x64x2x1 sw128", 4, {1024, 1024, 4, 8}, {2048, 2097152, 8388608}, {64, 64, 2, 1}, CU_TENSOR_MAP_SWIZZLE_128B, 8},
         {"4D 64x64x4x1 sw128", 4, {1024, 1024, 4, 8}, {2048, 2097152, 8388608}, {64, 64, 4, 1}, CU_TENSOR_MAP_SWIZZLE_128B, 8},
     };
+    {  // DRAM streaming: 2-D view (64 elems, rows) of the 2 GiB buffer; each CTA streams its own rows
+        for (int boxrows : {128, 256}) {
+            CUtensorMap m;
+            cuuint64_t dims[2] = {64, (cuuint64_t)(big_bytes / 128)};
+            cuuint64_t strides[1] = {128};
+            cuuint32_t box[2] = {64, (cuuint32_t)boxrows};
+            cuuint32_t es[2] = {1, 1};
+            CUresult r = enc(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, big, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                             CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+            if (r != CUDA_SUCCESS) { printf("dram encode failed\n"); return 1; }
+            int box_bytes = 128 * boxrows;
+            const int iters = 600;  // 600 boxes per CTA
+            int ncoord = (int)((big_bytes / 128) / 256 - 1);  // box index c -> rows c*256 (disjoint per CTA)
+            for (int stages : {4, 8, 12}) {
+                size_t smem = (size_t)stages * box_bytes + 1024;
+                if (smem > 227 * 1024) continue;
+                void* kfn = stages == 4 ? (void*)tma_loop<2, 4, 1> : stages == 8 ? (void*)tma_loop<2, 8, 1> : (void*)tma_loop<2, 12, 1>;
+                CK(cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                void* args[] = {&m, &box_bytes, (void*)&iters, &ncoord, &out};
+                cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+                cudaEventRecord(e0);
+                CK(cudaLaunchKernel(kfn, nsm, 128, args, smem, 0));
+                cudaEventRecord(e1);
+                CK(cudaDeviceSynchronize());
+                float ms; cudaEventElapsedTime(&ms, e0, e1);
+                std::vector<unsigned long long> h(148);
+                CK(cudaMemcpy(h.data(), out, 148 * 8, cudaMemcpyDeviceToHost));
+                double avg = 0; for (auto v : h) avg += v; avg /= 148;
+                printf("DRAM stream box %d B stages %2d : %6.1f B/cycle/SM  total %.0f GB/s\n", box_bytes, stages,
+                       (double)box_bytes * iters / avg, (double)box_bytes * iters * nsm / (ms * 1e6));
+            }
+        }
+    }
     for (auto& c : cases) {
         CUtensorMap m;
         cuuint32_t es[4] = {1, 1, 1, 1};
