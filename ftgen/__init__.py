@@ -87,6 +87,15 @@ def stacked_inputs(batch, seq, hidden, depth, seed, dtype="bf16", scale=1.0):
     )
 
 
+def linear_rnn_inputs(batch, seq, hidden, depth, seed, dtype="bf16", scale=1.0):
+    """Inputs of ft_stacked_rnn_fwd (Listing 1): x [B][T][H], W [D][H][H]."""
+    r = scale / np.sqrt(hidden)
+    return dict(
+        x=_draw(seed, S_X, (batch, seq, hidden), 1.0, dtype),
+        W=_draw(seed, S_W, (depth, hidden, hidden), r, dtype),
+    )
+
+
 def grid_inputs(batch, len_x, len_y, hidden, depth, seed, dtype="bf16", scale=1.0):
     """Inputs of ft_grid_rnn_fwd: x [B][Lx][H], ys [B][Ly][H], W [D][2][4][H][H],
     U [D][2][4][2H][H], b [D][2][4][H]."""

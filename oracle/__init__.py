@@ -42,7 +42,7 @@ def lib():
         build()
         _lib = ctypes.CDLL(LIB_PATH)
         for sfx in ("f64", "f32"):
-            for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell"):
+            for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell", "stacked_rnn"):
                 fn = getattr(_lib, f"ft_oracle_{name}_{sfx}")
                 fn.restype = ctypes.c_int if name != "lstm_cell" else None
     return _lib
@@ -154,3 +154,17 @@ def lstm_cell(a, W4, hp, U4, b4, cp, precision="f64"):
     getattr(lib(), f"ft_oracle_lstm_cell_{precision}")(
         H, _p(a), a.shape[0], _p(W4), _p(hp), Kh, _p(U4), _p(b4), _p(cp), _p(h), _p(c), _p(z))
     return h, c
+
+
+def stacked_rnn(x, W, precision="f64"):
+    """Stacked linear RNN oracle (Listing 1): y[d][t] = a @ W[d] + y[d][t-1].
+    x [B][T][H], W [D][H][H] → ysss [B][D][T][H]."""
+    dt = _prec(precision)
+    B, T, H = x.shape
+    D = W.shape[0]
+    x, W = _c(x, dt), _c(W, dt)
+    ys = np.empty((B, D, T, H), dt)
+    rc = getattr(lib(), f"ft_oracle_stacked_rnn_{precision}")(B, T, H, D, _p(x), _p(W), _p(ys))
+    if rc:
+        raise RuntimeError(f"oracle stacked_rnn failed: {rc}")
+    return ys

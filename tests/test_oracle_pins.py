@@ -344,3 +344,27 @@ def test_generator_is_counter_based_and_bf16_exact():
     p = ftgen.stacked_inputs(2, 3, 64, 2, 5, "bf16")
     assert np.max(np.abs(p["W"])) <= 1 / 8 and np.max(np.abs(p["x"])) <= 1
     ftgen.bf16_bits(p["W"])
+
+
+# --------------------------------------------------------------------------- P13 (Listing 1)
+@pytest.mark.parametrize("B,T,H,D", [(2, 6, 8, 3), (1, 9, 4, 1), (3, 4, 16, 5)])
+def test_p13_linear_rnn_closed_form(B, T, H, D):
+    """P13 (closed form): Listing 1's stacked RNN y[d][t] = a@W[d] + y[d][t-1] (L151–L165) is
+    linear: with C the T×T lower-triangular ones matrix (the time scanl with s0 = 0),
+    Y^(d) = C · Y^(d-1) · W_d, so Y^(D) = C^D · X · W_1 ⋯ W_D for every batch row."""
+    p = ftgen.linear_rnn_inputs(B, T, H, D, 21, "f32", scale=1.0)
+    ys = oracle.stacked_rnn(p["x"], p["W"])
+    C = np.tril(np.ones((T, T)))
+    for b in range(B):
+        Y = p["x"][b].astype(np.float64)
+        for d in range(D):
+            Y = C @ Y @ p["W"][d].astype(np.float64)
+            np.testing.assert_allclose(ys[b, d], Y, rtol=1e-12, atol=1e-12)
+
+
+def test_p13b_linear_rnn_layer_one_is_cumsum_of_projection():
+    """P13(b): one layer is the running sum over time (numpy cumsum) of x @ W (L159–L165)."""
+    p = ftgen.linear_rnn_inputs(2, 7, 8, 1, 22, "f32")
+    ys = oracle.stacked_rnn(p["x"], p["W"])
+    ref = np.cumsum(p["x"].astype(np.float64) @ p["W"][0].astype(np.float64), axis=1)
+    np.testing.assert_allclose(ys[:, 0], ref, rtol=1e-13, atol=1e-13)
