@@ -4,4 +4,4 @@ The product is libft.so (C ABI, include/ft.h) built from csrc/ for sm_100a; `ft`
 ctypes binding.  This package never imports oracle/ (the CPU test oracle).
 """
 from . import ft  # noqa: F401
-from .ft import dilated_rnn, grid_rnn, stacked_lstm  # noqa: F401
+from .ft import dilated_rnn, grid_rnn, stacked_lstm, stacked_rnn  # noqa: F401

@@ -30,7 +30,7 @@ size_t elem_size(ft_dtype dt) { return dt == FT_BF16 ? 2 : 4; }
 
 // Build the launch problem; returns OK or INVALID/UNSUPPORTED with g_last_error set.
 ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int* dil,
-                       ft_dtype dt, ft::Problem* p) {
+                       ft_dtype dt, ft::Problem* p, int cell = ft::CELL_LSTM) {
     if (dt != FT_F32 && dt != FT_BF16) return fail(FT_ERR_INVALID_ARGUMENT, "unknown dtype");
     if (B <= 0 || L0 <= 0 || L1 <= 0 || H <= 0 || D <= 0)
         return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
@@ -49,6 +49,7 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
 
     std::memset(p, 0, sizeof(*p));
     p->kind = kind;
+    p->cell = cell;
     p->B = B;
     p->H = H;
     p->D = D;
@@ -62,8 +63,11 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         // a5 weight residency: when every layer's weights fit in about half of the 126 MB L2
         // they are kept there across time steps (EVICT_LAST); otherwise they stream (EVICT_FIRST)
         // — a 256 MiB weight set cannot be resident, each diagonal re-reads it.
-        const double wbytes = (double)D * p->naxes * 4.0 * H * ((double)H + (kind == ft::KIND_SEQ ? H : 2.0 * H)) *
-                              (dt == FT_BF16 ? 2 : 4);
+        const double wbytes =
+            cell == ft::CELL_LINEAR
+                ? (double)D * H * H * (dt == FT_BF16 ? 2 : 4)
+                : (double)D * p->naxes * 4.0 * H * ((double)H + (kind == ft::KIND_SEQ ? H : 2.0 * H)) *
+                      (dt == FT_BF16 ? 2 : 4);
         p->resident_layers = wbytes <= 64.0 * 1024 * 1024 ? D : 0;
         const char* env = getenv("FT_L2_RESIDENT_LAYERS");  // tuning override
         if (env) p->resident_layers = atoi(env);
@@ -71,6 +75,7 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         p->debug = dbg ? atoi(dbg) : 0;
     }
     p->BNU = dt == FT_BF16 ? ft::BF16_BNU : ft::F32_BNU;
+    if (cell == ft::CELL_LINEAR && dt == FT_BF16) p->BNU = 4 * ft::BF16_BNU;  // 256 units per tile
     p->MB = (B + p->BM - 1) / p->BM;
     p->NT = (H + p->BNU - 1) / p->BNU;
     p->ncells = (long long)D * L0 * L1;
@@ -312,6 +317,36 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("D2H: ") + cudaGetErrorString(e));
     return FT_OK;
+}
+
+FT_API size_t ft_stacked_rnn_workspace_size(int batch, int seq, int hidden, int depth, ft_dtype dt) {
+    if (depth <= 0 || depth > FT_MAX_DEPTH) return 0;
+    int ones[FT_MAX_DEPTH];
+    for (int d = 0; d < depth; ++d) ones[d] = 1;
+    ft::Problem p;
+    if (make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, ones, dt, &p, ft::CELL_LINEAR) != FT_OK)
+        return 0;
+    return plan_workspace(p, dt, true).total;
+}
+
+FT_API ft_status ft_stacked_rnn_fwd(int batch, int seq, int hidden, int depth, ft_dtype dt,
+                                    const void* x, const void* W, void* ys, void* workspace,
+                                    size_t workspace_bytes, void* stream) {
+    if (depth <= 0) return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    if (depth > FT_MAX_DEPTH) return fail(FT_ERR_UNSUPPORTED, "depth > FT_MAX_DEPTH");
+    int ones[FT_MAX_DEPTH];
+    for (int d = 0; d < depth; ++d) ones[d] = 1;
+    ft::Problem p;
+    ft_status st = make_problem(ft::KIND_SEQ, batch, seq, 1, hidden, depth, ones, dt, &p, ft::CELL_LINEAR);
+    if (st != FT_OK) return st;
+    REQUIRE_PTR(x, "x");
+    REQUIRE_PTR(W, "W");
+    REQUIRE_PTR(ys, "ys");
+    ft::Tensors t;
+    t.x = x;
+    t.W = W;
+    t.h_all = ys;  // Listing 1's ysss [N, D, L] is the SSA buffer itself
+    return run(p, dt, t, workspace, workspace_bytes, stream);
 }
 
 FT_API size_t ft_dilated_rnn_workspace_size(int batch, int seq, int hidden, int depth,

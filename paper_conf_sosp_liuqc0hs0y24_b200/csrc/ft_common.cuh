@@ -23,10 +23,14 @@
 namespace ft {
 
 enum Kind : int { KIND_SEQ = 0 /* stacked + dilated */, KIND_GRID = 1 };
+// Cell function: the LSTM of Listing 2 (L607–L615) or the linear cell y = x@w + s of Listing 1
+// (L165; one weight matrix, no gates, the recurrent term is an addition of the previous output).
+enum CellType : int { CELL_LSTM = 0, CELL_LINEAR = 1 };
 
 // One launch's problem.  All sizes in elements.
 struct Problem {
     int kind;
+    int cell;            // CellType
     int B, H, D;
     int L0, L1;          // KIND_SEQ: L0 = seq, L1 = 1.  KIND_GRID: L0 = len_x, L1 = len_y.
     int naxes;           // 1 (seq) or 2 (grid)
@@ -197,7 +201,8 @@ FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
         seg[0] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0}
                             : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0};
         const int s = p.dil[c.d];
-        seg[1] = Segment{c.i >= s ? SRC_H : SRC_NONE, c.i >= s ? h_row(p, c.d, c.i - s, 0, 0) : 0,
+        const bool rec = c.i >= s && p.cell == CELL_LSTM;  // the linear cell has no h@U term
+        seg[1] = Segment{rec ? SRC_H : SRC_NONE, rec ? h_row(p, c.d, c.i - s, 0, 0) : 0,
                          W_REC, c.d, 0};
         seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0};
     } else {

@@ -168,8 +168,11 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         const int nchunks = ns * kchunks;
         const int npre = nchunks < C::STAGES ? nchunks : C::STAGES;
         const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
-        const int bn = fixed ? 0 : tl.n * BNU;
-        const int bg = (int)rank * C::GATES;
+        // weight box: LSTM (n = 64-unit slab, gate atoms), linear cell (n_lo = 0, 64-unit atoms
+        // n_hi = 4 per 256-unit tile)
+        const bool lin = P.cell == CELL_LINEAR;
+        const int bn = (fixed || lin) ? 0 : tl.n * BNU;
+        const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
         FT_TR_DECL;
         int first_stage = stage;
         int si = 0, kc = 0;
@@ -318,9 +321,97 @@ constexpr int EPI_WARPS = 8;
 constexpr int EPI_THREADS = EPI_WARPS * 32;
 constexpr int EPI_UNITS = BNU / 2;  // units per thread
 
+// Listing 1's linear cell: y = z + s, s = the previous step's output (fp32 ring), 0 at t = 0.
+// The 256 accumulator columns are 256 consecutive units; warp half h takes columns h*128 ...
+template <int CG>
+__device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tensors& T,
+                                                    uint32_t tmem_base, uint64_t* tfull,
+                                                    uint64_t* tempty, uint32_t rank) {
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const int q = warp & 3, half = (warp - 2) >> 2, row = q * 32 + lane;
+    const bool leader_thread = (threadIdx.x == 64);
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    Cursor cur = cursor_begin();
+    const int target = flag_target(P);
+    __nv_bfloat16* ys = (__nv_bfloat16*)T.h_all;
+    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    for (long long tile = first; tile < P.ntiles; tile += stride) {
+        const TileId tl = decode_tile(P, cur, tile);
+        const Cell c = tl.cell;
+        int ci = 0, cj = 0;
+        const long long cprod = c_producer(P, tl, &ci, &cj);
+        const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
+        const bool valid = b < P.B;
+        const int n0 = tl.n * 4 * BNU + half * 2 * BNU;
+        if (cprod >= 0 && leader_thread) wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
+        named_bar_sync(1, EPI_THREADS);
+        mbar_wait(&tfull[acc], acc_phase);
+        tc_fence_after();
+        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
+                               (uint32_t)(half * 2 * BNU);
+        const int row_h = h_row(P, c.d, c.i, c.j, 0);
+#pragma unroll 1
+        for (int u0 = 0; u0 < 2 * BNU; u0 += 16) {
+            __syncwarp();
+            float z[16];
+            tmem_ld_32x32b_x16(tbase + u0, z);
+            tmem_wait_ld();
+            if (u0 + 16 == 2 * BNU) {
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) {
+                    if constexpr (CG == 1)
+                        mbar_arrive(&tempty[acc]);
+                    else
+                        mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[acc]), 0));
+                }
+            }
+            const int n = n0 + u0;
+            if (!valid || n >= P.H) continue;
+            if (cprod >= 0) {
+                const float4* src = reinterpret_cast<const float4*>(T.c_ring + c_ring_index(P, c.d, ci, cj, 0, b, n));
+#pragma unroll
+                for (int v = 0; v < 4; ++v) {
+                    const float4 t4 = __ldcg(src + v);
+                    z[4 * v] += t4.x;
+                    z[4 * v + 1] += t4.y;
+                    z[4 * v + 2] += t4.z;
+                    z[4 * v + 3] += t4.w;
+                }
+            }
+            uint4 hp[2];
+#pragma unroll
+            for (int w = 0; w < 2; ++w)
+                hp[w] = make_uint4(pack_bf16x2(z[8 * w + 0], z[8 * w + 1]), pack_bf16x2(z[8 * w + 2], z[8 * w + 3]),
+                                   pack_bf16x2(z[8 * w + 4], z[8 * w + 5]), pack_bf16x2(z[8 * w + 6], z[8 * w + 7]));
+            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, 0, b, n));
+#pragma unroll
+            for (int v = 0; v < 4; ++v) __stcg(cdst + v, make_float4(z[4 * v], z[4 * v + 1], z[4 * v + 2], z[4 * v + 3]));
+            uint4* hdst = reinterpret_cast<uint4*>((__nv_bfloat16*)T.hb + hb_row(P, row_h, n / 64, b) * 64 + (n % 64));
+            __stcg(hdst, hp[0]);
+            __stcg(hdst + 1, hp[1]);
+            uint4* ydst = reinterpret_cast<uint4*>(ys + h_all_index(P, c, 0, b, n));
+            ydst[0] = hp[0];
+            ydst[1] = hp[1];
+        }
+        named_bar_sync(1, EPI_THREADS);
+        if (leader_thread) {
+            __threadfence();
+            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+        }
+        acc ^= 1;
+        if (acc == 0) acc_phase ^= 1;
+    }
+}
+
 template <int CG>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
                                              uint64_t* tfull, uint64_t* tempty, uint32_t rank) {
+    if (P.cell == CELL_LINEAR) {
+        run_epilogue_linear<CG>(P, T, tmem_base, tfull, tempty, rank);
+        return;
+    }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3;                 // TMEM lane quadrant this warp may access
     const int half = (warp - 2) >> 2;       // which 32 units of the tile
@@ -629,9 +720,26 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
                     p.kind == KIND_GRID ? p.L1 : p.L0, p.B, err))
         return cudaErrorInvalidValue;
     if (!encode_blocked(enc, &M.h, t.hb, hb_rows_total(p), err)) return cudaErrorInvalidValue;
-    if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, err)) return cudaErrorInvalidValue;
-    if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, err))
-        return cudaErrorInvalidValue;
+    if (p.cell == CELL_LINEAR) {
+        // W [D][H][H] as (64 n_lo, k, H/64 n_hi, d): a box of 4 (or 2) 64-unit atoms is the
+        // 256-unit N tile of one 64-deep K chunk — the same SMEM layout as the LSTM gate atoms
+        const cuuint64_t dims[4] = {64, (cuuint64_t)p.H, (cuuint64_t)(p.H / 64), (cuuint64_t)p.D};
+        const cuuint64_t strides[3] = {(cuuint64_t)p.H * 2, 128, (cuuint64_t)p.H * p.H * 2};
+        const cuuint32_t box[4] = {64, (cuuint32_t)BK, (cuuint32_t)C::GATES, 1};
+        const cuuint32_t es[4] = {1, 1, 1, 1};
+        CUresult r = enc(&M.W, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(t.W), dims, strides,
+                         box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) {
+            if (err) *err = "cuTensorMapEncodeTiled(linear weight) failed: " + std::to_string((int)r);
+            return cudaErrorInvalidValue;
+        }
+        M.U = M.W;
+    } else {
+        if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, err)) return cudaErrorInvalidValue;
+        if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, err))
+            return cudaErrorInvalidValue;
+    }
 
     int dev = 0, nsm = 0;
     cudaError_t e = cudaGetDevice(&dev);

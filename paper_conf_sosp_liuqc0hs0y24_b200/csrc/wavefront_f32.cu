@@ -59,10 +59,12 @@ wavefront_f32_kernel(const __grid_constant__ Problem P, const __grid_constant__ 
         const int n = n0 + u;
         const bool nvalid = n < P.H;
         const int slice_b = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
+        const bool lstm = P.cell == CELL_LSTM;
+        const int ng = lstm ? 4 : 1;  // gate blocks of the weight slice (linear cell: one matrix)
         float acc[4][4];
 #pragma unroll
         for (int g = 0; g < 4; ++g) {
-            const float bv = nvalid ? __ldg(T.b + ((long long)slice_b * 4 + g) * P.H + n) : 0.f;
+            const float bv = (nvalid && lstm) ? __ldg(T.b + ((long long)slice_b * 4 + g) * P.H + n) : 0.f;
 #pragma unroll
             for (int r = 0; r < 4; ++r) acc[r][g] = bv;
         }
@@ -88,8 +90,8 @@ wavefront_f32_kernel(const __grid_constant__ Problem P, const __grid_constant__ 
                     const int uu = e % BNU, kk = (e / BNU) % KC, g = e / (BNU * KC);
                     const int k = k0 + kk, nn = n0 + uu;
                     float v = 0.f;
-                    if (k < P.H && nn < P.H)
-                        v = __ldg(Wt + (((long long)seg[s].slice * 4 + g) * krows + seg[s].krow0 + k) * P.H + nn);
+                    if (k < P.H && nn < P.H && g < ng)
+                        v = __ldg(Wt + (((long long)seg[s].slice * ng + g) * krows + seg[s].krow0 + k) * P.H + nn);
                     sm.w[g][kk][uu] = v;
                 }
                 __syncthreads();
@@ -116,6 +118,13 @@ wavefront_f32_kernel(const __grid_constant__ Problem P, const __grid_constant__ 
         for (int r = 0; r < 4; ++r) {
             const int b = m0 + rg * 4 + r;
             if (b >= P.B || !nvalid) continue;
+            if (!lstm) {  // Listing 1: y = x@w + s (s = the previous step's output, 0 at t = 0)
+                const float sp = (cprod >= 0) ? __ldcg(T.c_ring + c_ring_index(P, c.d, ci, cj, 0, b, n)) : 0.f;
+                const float yv = acc[r][0] + sp;
+                __stcg((float*)T.h_all + h_all_index(P, c, 0, b, n), yv);
+                __stcg(T.c_ring + c_ring_index(P, c.d, c.i, c.j, 0, b, n), yv);
+                continue;
+            }
             const float ig = 1.f / (1.f + expf(-acc[r][0]));
             const float fg = 1.f / (1.f + expf(-acc[r][1]));
             const float og = 1.f / (1.f + expf(-acc[r][2]));

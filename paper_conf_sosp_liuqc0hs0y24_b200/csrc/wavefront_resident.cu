@@ -351,7 +351,7 @@ cudaError_t launch_resident_t(const Problem& p, const Tensors& t, cudaStream_t s
 // Which resident slab width fits (0 = the weights cannot be resident): stacked only (every
 // dilation 1), batch <= 128, one CTA per (layer, slab) on distinct SMs, slab + A ring <= 227 KB.
 int resident_bnu(const Problem& p, int nsm) {
-    if (p.kind != KIND_SEQ || p.B > RROWS || p.H % 64 != 0) return 0;
+    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM || p.B > RROWS || p.H % 64 != 0) return 0;
     for (int d = 0; d < p.D; ++d)
         if (p.dil[d] != 1) return 0;
     const size_t cap = 227 * 1024;

@@ -28,6 +28,7 @@ EXPORTS = (
     "ft_version", "ft_status_string", "ft_last_error",
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
     "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
+    "ft_stacked_rnn_workspace_size", "ft_stacked_rnn_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells",
@@ -71,6 +72,10 @@ def lib():
         L.ft_stacked_lstm_hostio_workspace_size.argtypes = [_c_int] * 5
         L.ft_stacked_lstm_fwd_hostio.restype = _c_int
         L.ft_stacked_lstm_fwd_hostio.argtypes = [_c_int] * 5 + [_c_vp] * 7 + [_c_vp, _c_size, _c_vp]
+        L.ft_stacked_rnn_workspace_size.restype = _c_size
+        L.ft_stacked_rnn_workspace_size.argtypes = [_c_int] * 5
+        L.ft_stacked_rnn_fwd.restype = _c_int
+        L.ft_stacked_rnn_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 3 + [_c_vp, _c_size, _c_vp]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         _lib = L
@@ -125,6 +130,16 @@ def ft_stacked_lstm_fwd_hostio(batch, seq, hidden, depth, dt, x_host, W, U, b, y
     return lib().ft_stacked_lstm_fwd_hostio(batch, seq, hidden, depth, dt, x_host, W, U, b,
                                             y_host, h_n_host, c_n_host, workspace,
                                             workspace_bytes, stream)
+
+
+def ft_stacked_rnn_workspace_size(batch, seq, hidden, depth, dt):
+    return lib().ft_stacked_rnn_workspace_size(batch, seq, hidden, depth, dt)
+
+
+def ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace, workspace_bytes,
+                       stream) -> int:
+    return lib().ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace,
+                                    workspace_bytes, stream)
 
 
 def ft_dilated_rnn_fwd(batch, seq, hidden, depth, dilations, dt, x, W, U, b, y, h_n, c_n, h_all,
@@ -261,3 +276,18 @@ def grid_rnn(x, ys, W, U, b, want_all=False, stream=None, workspace=None):
     if want_all:
         r.update(h_all=h_all, c_all=c_all)
     return r
+
+
+def stacked_rnn(x, W, stream=None, workspace=None):
+    """Listing 1's stacked linear RNN (y = x@w + s) through the C ABI.
+    x [B][T][H] (bf16 / fp32 CUDA), W [D][H][H] → ys [B][D][T][H] (every layer's output)."""
+    torch = _torch()
+    B, T, H = x.shape
+    D = W.shape[0]
+    dt = _dt(x)
+    ys = torch.empty((B, D, T, H), dtype=x.dtype, device=x.device)
+    nbytes = ft_stacked_rnn_workspace_size(B, T, H, D, dt)
+    ws = (workspace or Workspace()).get(nbytes, x.device)
+    check(ft_stacked_rnn_fwd(B, T, H, D, dt, _ptr(x), _ptr(W), _ptr(ys), ws.data_ptr(), ws.numel(),
+                             _stream_ptr(stream)))
+    return ys

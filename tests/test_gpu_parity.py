@@ -208,3 +208,22 @@ def test_bf16_C5_sampled_rows():
     rows = ftgen.sample_rows(c["batch"], 0, 3)[:4]
     ref = oracle.grid_rnn(g["x"][rows], g["ys"][rows], g["W"], g["U"], g["b"])
     _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n"), rows=rows, ctx="C5")
+
+
+# ------------------------------------------------------------------------- Listing 1 (NEXT-3)
+@pytest.mark.parametrize("B,T,H,D", [(3, 5, 16, 2), (33, 4, 40, 3), (1, 1, 8, 1)])
+def test_f32_linear_rnn(B, T, H, D):
+    """Listing 1 (L140–L166) y = x@w + s on the fp32 wavefront vs the oracle (max abs 1e-4)."""
+    p = ftgen.linear_rnn_inputs(B, T, H, D, 808 + H, "f32")
+    ys = ft.stacked_rnn(dev(p["x"], torch.float32), dev(p["W"], torch.float32))
+    torch.cuda.synchronize()
+    _check({"ys": ys}, {"ys": oracle.stacked_rnn(p["x"], p["W"])}, torch.float32, ("ys",), ctx="f32 linear")
+
+
+@pytest.mark.parametrize("B,T,H,D", [(4, 6, 256, 3), (130, 5, 512, 2), (256, 7, 320, 4), (9, 1, 64, 1)])
+def test_bf16_linear_rnn(B, T, H, D):
+    """Listing 1 on the tcgen05 wavefront (1-CTA and CTA-pair tiles, partial 256-unit tiles)."""
+    p = ftgen.linear_rnn_inputs(B, T, H, D, 909 + H, "bf16")
+    ys = ft.stacked_rnn(dev(p["x"], torch.bfloat16), dev(p["W"], torch.bfloat16))
+    torch.cuda.synchronize()
+    _check({"ys": ys}, {"ys": oracle.stacked_rnn(p["x"], p["W"])}, torch.bfloat16, ("ys",), ctx="bf16 linear")
