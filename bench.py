@@ -132,6 +132,19 @@ class ClockSampler:
 
 
 # ----------------------------------------------------------------------------- CPU oracle
+def host_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def pin_oracle_threads():
+    # torchrun exports OMP_NUM_THREADS=1; the CPU baseline uses every host core it may run on.
+    # Must run before oracle/liboracle.so is first loaded (OpenMP reads it at initialisation).
+    os.environ["OMP_NUM_THREADS"] = str(host_cores())
+
+
 def oracle_rate(p, rows, tsteps=None):
     """Time the CPU oracle (f32 instantiation, as it stands) on `rows` batch rows of the
     workload, optionally only the first `tsteps` time steps.  Returns (seconds, sequences)."""
@@ -145,6 +158,7 @@ def oracle_rate(p, rows, tsteps=None):
 
 
 def cpu_baseline(p):
+    pin_oracle_threads()
     import oracle
     n = oracle.num_threads()
     dt, seqs = oracle_rate(p, n)
@@ -172,6 +186,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    pin_oracle_threads()
     import oracle
     c, p = make_inputs(0)
     nthr = oracle.num_threads()
@@ -218,10 +233,22 @@ def run_ours(args):
     if world != args.gpus and world > 1:
         print(f"warning: WORLD_SIZE={world} != --gpus {args.gpus}", file=sys.stderr)
     n_gpus = world
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    backend = os.environ.get("FT_DIST_BACKEND", "nccl")  # gloo: exercise the multi-rank path on 1 GPU
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(backend)
+
+    def max_over_ranks(v):
+        if world == 1:
+            return v
+        t = torch.tensor([v], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
 
     c, p = make_inputs(rank)
     B, T, H, D = c["batch"], c["seq"], c["hidden"], c["depth"]
@@ -268,10 +295,7 @@ def run_ours(args):
     clocks = sampler.stop()
     elapsed_ms = t0.elapsed_time(t1)
     call_ms = [s.elapsed_time(e) for s, e in ev]
-    if world > 1:
-        t = torch.tensor([elapsed_ms], device=dev, dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        elapsed_ms = float(t.item())
+    elapsed_ms = max_over_ranks(elapsed_ms)
     ms_per_step = elapsed_ms / args.steps
     value = n_gpus * B * args.steps / (elapsed_ms / 1e3)
 
@@ -317,11 +341,7 @@ def run_ours(args):
             e2e_step()
         a1.record(stream)
         torch.cuda.synchronize()
-        e_ms = a0.elapsed_time(a1)
-        if world > 1:
-            t = torch.tensor([e_ms], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            e_ms = float(t.item())
+        e_ms = max_over_ranks(a0.elapsed_time(a1))
         # sanity: the host result equals the device-path result of the same batch
         ok = bool(torch.equal(y_h.to(dev), outs["y"]))
         e2e = {"value": n_gpus * B * ke / (e_ms / 1e3), "unit": UNIT,

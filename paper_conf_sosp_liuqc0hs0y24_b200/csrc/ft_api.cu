@@ -103,7 +103,8 @@ struct WsPlan {
 WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     WsPlan w{};
     w.flags_off = 0;
-    w.flags_bytes = round_up((size_t)p.ncells * p.MB * sizeof(int), 256);
+    // tile-granular counters (bf16 streaming kernel) — also covers the cell-granular protocols
+    w.flags_bytes = round_up((size_t)p.ncells * p.naxes * p.MB * p.NT * sizeof(int), 256);
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
     w.hall_off = w.ring_off + w.ring_bytes;

@@ -108,8 +108,17 @@ FT_HD long long cell_lin(const Problem& p, int d, int i, int j) {
 
 FT_HD int tiles_per_cell(const Problem& p) { return p.naxes * p.MB * p.NT; }
 
-// Flags: one int per (cell, m-block); complete when it reaches naxes * NT * flag_mult.
+// Flags: one int per (cell, m-block); complete when it reaches naxes * NT * flag_mult
+// (cell-granular protocol of the fp32 kernel).
 FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
+
+// Tile-granular protocol of the bf16 streaming kernel: one counter per (cell, axis, m-block,
+// N-tile), complete when it reaches flag_mult (the CTAs of the tile).  A consumer's K-chunk kc
+// only needs the producer's units [kc*64, kc*64+64) — one N-tile — so consecutive diagonals
+// pipeline at tile granularity instead of waiting for whole cells.
+FT_HD long long tile_flag(const Problem& p, long long cell, int axis, int m, int n) {
+    return ((cell * p.naxes + axis) * p.MB + m) * (long long)p.NT + n;
+}
 
 // Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).
 struct Cursor {
@@ -178,6 +187,8 @@ struct Segment {
     int wsel;   // WSel
     int slice;  // weight slice: d (seq) or d*2+axis (grid)
     int krow0;  // first K row inside the weight slice (grid U: 0 for h^x, H for h^y)
+    int scell;  // SRC_H: linear index of the cell that produced these activations
+    int saxis;  // SRC_H: its axis (grid), 0 otherwise
 };
 
 // rows per batch row of h_all
@@ -198,23 +209,25 @@ FT_HD int u_krows(const Problem& p) { return p.kind == KIND_SEQ ? p.H : 2 * p.H;
 FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
     const Cell& c = tl.cell;
     if (p.kind == KIND_SEQ) {
-        seg[0] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0}
-                            : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0};
+        seg[0] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0, -1, 0}
+                            : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0,
+                                      (int)cell_lin(p, c.d - 1, c.i, 0), 0};
         const int s = p.dil[c.d];
         const bool rec = c.i >= s && p.cell == CELL_LSTM;  // the linear cell has no h@U term
         seg[1] = Segment{rec ? SRC_H : SRC_NONE, rec ? h_row(p, c.d, c.i - s, 0, 0) : 0,
-                         W_REC, c.d, 0};
-        seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0};
+                         W_REC, c.d, 0, rec ? (int)cell_lin(p, c.d, c.i - s, 0) : -1, 0};
+        seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0, -1, 0};
     } else {
         const int a = tl.axis, sl = c.d * 2 + a;
         if (c.d == 0)
-            seg[0] = Segment{a == 0 ? SRC_X : SRC_YS, a == 0 ? c.i : c.j, W_IN, sl, 0};
+            seg[0] = Segment{a == 0 ? SRC_X : SRC_YS, a == 0 ? c.i : c.j, W_IN, sl, 0, -1, 0};
         else
-            seg[0] = Segment{SRC_H, h_row(p, c.d - 1, c.i, c.j, a), W_IN, sl, 0};
+            seg[0] = Segment{SRC_H, h_row(p, c.d - 1, c.i, c.j, a), W_IN, sl, 0,
+                             (int)cell_lin(p, c.d - 1, c.i, c.j), a};
         seg[1] = Segment{c.i > 0 ? SRC_H : SRC_NONE, c.i > 0 ? h_row(p, c.d, c.i - 1, c.j, 0) : 0,
-                         W_REC, sl, 0};
+                         W_REC, sl, 0, c.i > 0 ? (int)cell_lin(p, c.d, c.i - 1, c.j) : -1, 0};
         seg[2] = Segment{c.j > 0 ? SRC_H : SRC_NONE, c.j > 0 ? h_row(p, c.d, c.i, c.j - 1, 1) : 0,
-                         W_REC, sl, p.H};
+                         W_REC, sl, p.H, c.j > 0 ? (int)cell_lin(p, c.d, c.i, c.j - 1) : -1, 1};
     }
     return 1 + (seg[1].src != SRC_NONE) + (seg[2].src != SRC_NONE);
 }
@@ -317,6 +330,18 @@ __device__ __forceinline__ int ld_acquire_gpu(const int* p) {
     int v;
     asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
+}
+
+__device__ __forceinline__ int ld_relaxed_gpu(const int* p) {
+    int v;
+    asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// acquire fence: with the relaxed loads before it that observed released values, this gives
+// those loads acquire semantics (fence-based synchronization of the PTX memory model)
+__device__ __forceinline__ void fence_acq_rel_gpu() {
+    asm volatile("fence.acq_rel.gpu;" ::: "memory");
 }
 
 __device__ __forceinline__ void red_release_gpu_add(int* p, int v) {

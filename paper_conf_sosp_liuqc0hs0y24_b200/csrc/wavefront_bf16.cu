@@ -19,9 +19,11 @@
 //           issues M256 N256 K16 MMAs reading both CTAs' shared memory, so each weight tile is
 //           fetched once per cell for the whole 256-row batch and per-CTA weight traffic halves.
 //
-// Warp roles (320 threads per CTA):
-//   warp 0      TMA producer: waits the tile's producer cells (readiness counters), then streams
-//               64-deep K-chunks of A and B into a STAGES-deep shared-memory ring (mbarriers).
+// Warp roles (352 threads per CTA):
+//   warp 0      weight TMA producer: streams the 64-deep K-chunks of B (no dependencies) into a
+//               STAGES-deep shared-memory ring (mbarriers), running ahead of the wavefront.
+//   warp 10     activation TMA producer: waits the tile's producer cells (readiness counters),
+//               then streams the matching K-chunks of A into the same ring slots.
 //   warp 1      MMA issuer (leader CTA): one thread issues tcgen05.mma into a double-buffered
 //               TMEM accumulator (2 x 256 fp32 columns) so tile n+1's MMAs overlap tile n's
 //               epilogue.
@@ -87,7 +89,7 @@ constexpr int BNU = BF16_BNU;  // 64 hidden units per tile
 constexpr int BN = 4 * BNU;    // 256 = UMMA N (i | f | o | ĝ)
 constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16
 constexpr int UK = 16;         // UMMA K for kind::f16
-constexpr int THREADS = 320;  // warp 0 TMA, warp 1 MMA, warps 2-9 epilogue
+constexpr int THREADS = 352;  // warp 0 weight TMA, 1 MMA, 2-9 epilogue, 10 activation TMA
 constexpr int TMEM_COLS = 2 * BN;  // double-buffered accumulator
 
 template <int CG>
@@ -126,6 +128,8 @@ __device__ __forceinline__ Segment pick(const Segment (&seg)[3], int i) {
     r.wsel = i == 0 ? seg[0].wsel : (i == 1 ? seg[1].wsel : seg[2].wsel);
     r.slice = i == 0 ? seg[0].slice : (i == 1 ? seg[1].slice : seg[2].slice);
     r.krow0 = i == 0 ? seg[0].krow0 : (i == 1 ? seg[1].krow0 : seg[2].krow0);
+    r.scell = i == 0 ? seg[0].scell : (i == 1 ? seg[1].scell : seg[2].scell);
+    r.saxis = i == 0 ? seg[0].saxis : (i == 1 ? seg[1].saxis : seg[2].saxis);
     return r;
 }
 
@@ -142,7 +146,13 @@ __device__ __forceinline__ void load_a(const Problem& P, const Maps& M, uint32_t
     }
 }
 
-template <int CG>
+// Two producer threads in different warps share the ring: the WEIGHT producer (no dependencies,
+// runs up to STAGES chunks ahead, i.e. the HBM weight stream never waits for the wavefront) and
+// the ACTIVATION producer (acquires the tile's producer cells, then loads A).  Each ring slot's
+// full barrier (in the leader CTA) takes one expect-tx arrival from each of the leader's two
+// producers; the peer CTA's producers only issue loads.  Splitting halves the serial TMA issue
+// work per thread (the role trace showed one thread issuing both was the limiter).
+template <int CG, bool kWeights>
 __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
                                              uint8_t* sA, uint8_t* sB, uint64_t* full,
                                              uint64_t* empty, uint32_t rank) {
@@ -158,7 +168,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const uint64_t pol_keep = policy_evict_last();
     const uint64_t pol_act = policy_evict_normal();
     const bool skipA = P.debug & 8, skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
-    const uint32_t tx = CG * ((skipA ? 0 : C::A_BYTES) + (skipB ? 0 : C::B_BYTES));
+    const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : (skipA ? 0 : CG * C::A_BYTES);
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
     FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
@@ -166,55 +176,43 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         Segment seg[3];
         const int ns = segments(P, tl, seg);
         const int nchunks = ns * kchunks;
-        const int npre = nchunks < C::STAGES ? nchunks : C::STAGES;
         const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
-        // weight box: LSTM (n = 64-unit slab, gate atoms), linear cell (n_lo = 0, 64-unit atoms
-        // n_hi = 4 per 256-unit tile)
         const bool lin = P.cell == CELL_LINEAR;
         const int bn = (fixed || lin) ? 0 : tl.n * BNU;
         const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
         FT_TR_DECL;
-        int first_stage = stage;
+        if constexpr (!kWeights) {
+            // the producer cells of this tile (Table 4 dependence vectors): one acquire each of
+            // their (cell, m-block) counters before any activation load of the tile
+            FT_TR_ADD(TR_TILES, 1);
+            long long prod[3];
+            producers(P, tl.cell, prod);
+            FT_TR_BEGIN();
+            if (!(P.debug & 1)) {
+#pragma unroll
+                for (int q = 0; q < 3; ++q)
+                    if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
+            }
+            FT_TR_END(TR_P_FLAG);
+            fence_proxy_async_global();
+        }
         int si = 0, kc = 0;
         for (int c = 0; c < nchunks; ++c) {
             const Segment sg = pick(seg, si);
-            FT_TR_BEGIN();
+            if constexpr (kWeights) FT_TR_BEGIN();
             mbar_wait(&empty[stage], phase ^ 1);
-            FT_TR_END(TR_P_EMPTY);
+            if constexpr (kWeights) FT_TR_END(TR_P_EMPTY);
             const uint32_t bar = full0 + 8u * (uint32_t)stage;
             if (rank == 0) mbar_arrive_expect_tx(&full[stage], tx);
-            if (!skipB) {
-                const CUtensorMap* bm = sg.wsel == W_IN ? &M.W : &M.U;
-                const uint64_t wpol = weight_layer(P, sg.slice) < P.resident_layers ? pol_keep : pol_stream;
-                tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
-                                          fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
-            }
-            if (c >= npre) {
+            if constexpr (kWeights) {
+                if (!skipB) {
+                    const CUtensorMap* bm = sg.wsel == W_IN ? &M.W : &M.U;
+                    const uint64_t wpol = weight_layer(P, sg.slice) < P.resident_layers ? pol_keep : pol_stream;
+                    tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
+                                              fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
+                }
+            } else {
                 if (!skipA) load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
-            } else if (c + 1 == npre) {
-                // dependencies (Table 4 vectors) of this tile, then the deferred A loads
-                long long prod[3];
-                const int np = producers(P, tl.cell, prod);
-                FT_TR_BEGIN();
-                if (!(P.debug & 1)) {
-#pragma unroll
-                    for (int q = 0; q < 3; ++q)
-                        if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
-                }
-                (void)np;
-                FT_TR_END(TR_P_FLAG);
-                FT_TR_ADD(TR_TILES, 1);
-                fence_proxy_async_global();
-                if (!skipA) {
-                    int ps = first_stage, psi = 0, pkc = 0;
-                    for (int cc = 0; cc < npre; ++cc) {
-                        const Segment sa = pick(seg, psi);
-                        load_a<CG>(P, M, sA0 + (uint32_t)(ps * C::A_BYTES), full0 + 8u * (uint32_t)ps,
-                                   sa, pkc, arow0, fixed, pol_act);
-                        if (++ps == C::STAGES) ps = 0;
-                        if (++pkc == kchunks) { pkc = 0; psi = next_segment(seg, psi); }
-                    }
-                }
             }
             if (++kc == kchunks) { kc = 0; si = next_segment(seg, si); }
             if (++stage == C::STAGES) {
@@ -223,7 +221,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             }
         }
     }
-    FT_TR_FLUSH(true);
+    FT_TR_FLUSH(true);  // the two producers fill disjoint slots
 }
 
 // ------------------------------------------------------------------------------ MMA issuer
@@ -344,7 +342,8 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
         const int n0 = tl.n * 4 * BNU + half * 2 * BNU;
-        if (cprod >= 0 && leader_thread) wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
+        if (cprod >= 0 && leader_thread)
+            wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
         named_bar_sync(1, EPI_THREADS);
         mbar_wait(&tfull[acc], acc_phase);
         tc_fence_after();
@@ -593,7 +592,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     FT_TR_BEGIN();
     if (threadIdx.x == 0) {
         for (int s = 0; s < C::STAGES; ++s) {
-            mbar_init(&full[s], 1);
+            mbar_init(&full[s], 2);  // the leader's weight + activation producers
             mbar_init(&empty[s], 1);
         }
         for (int a = 0; a < 2; ++a) {
@@ -615,9 +614,11 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == 0) {
-        if (lane == 0) run_producer<CG>(P, T, M, sA, sB, full, empty, rank);
+        if (lane == 0) run_producer<CG, true>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
         if (lane == 0 && rank == 0) run_mma<CG>(P, tmem_base, sA, sB, full, empty, tfull, tempty);
+    } else if (warp == 10) {
+        if (lane == 0) run_producer<CG, false>(P, T, M, sA, sB, full, empty, rank);
     } else {
         run_epilogue<CG>(P, T, tmem_base, tfull, tempty, rank);
     }
