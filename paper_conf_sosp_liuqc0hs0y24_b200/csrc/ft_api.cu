@@ -97,6 +97,7 @@ struct WsPlan {
     size_t flags_off, flags_bytes;
     size_t ring_off, ring_bytes;
     size_t hall_off, hall_bytes;
+    size_t xb_off, xb_bytes, yb_off, yb_bytes;  // bf16: inputs packed into the blocked layout
     size_t total;
 };
 
@@ -114,7 +115,13 @@ WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
         w.hall_bytes = h_all_provided
                            ? 0
                            : round_up((size_t)p.B * ft::h_rows(p) * p.H * elem_size(dt), 256);
-    w.total = w.hall_off + w.hall_bytes;
+    w.xb_off = w.hall_off + w.hall_bytes;
+    w.xb_bytes = dt == FT_BF16 ? round_up((size_t)p.L0 * p.H * ((size_t)p.MB * p.BM) * 2, 256) : 0;
+    w.yb_off = w.xb_off + w.xb_bytes;
+    w.yb_bytes = (dt == FT_BF16 && p.kind == ft::KIND_GRID)
+                     ? round_up((size_t)p.L1 * p.H * ((size_t)p.MB * p.BM) * 2, 256)
+                     : 0;
+    w.total = w.yb_off + w.yb_bytes;
     return w;
 }
 
@@ -145,9 +152,11 @@ ft_status run(const ft::Problem& p, ft_dtype dt, ft::Tensors t, void* workspace,
     uint8_t* ws = static_cast<uint8_t*>(workspace);
     t.flags = reinterpret_cast<int*>(ws + w.flags_off);
     t.c_ring = reinterpret_cast<float*>(ws + w.ring_off);
-    if (dt == FT_BF16)
+    if (dt == FT_BF16) {
         t.hb = ws + w.hall_off;
-    else if (!t.h_all)
+        t.xb = ws + w.xb_off;
+        t.yb = w.yb_bytes ? ws + w.yb_off : nullptr;
+    } else if (!t.h_all)
         t.h_all = ws + w.hall_off;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
     cudaError_t e = cudaMemsetAsync(t.flags, 0, w.flags_bytes, s);  // BK0: reset readiness flags

@@ -21,6 +21,8 @@ struct Tensors {
     float* c_n = nullptr;
     void* h_all = nullptr;   // f32 path: never NULL at launch (workspace stand-in); bf16: optional
     void* hb = nullptr;      // bf16 path: blocked SSA activations [h_rows][H/64][Bp][64] (workspace)
+    void* xb = nullptr;      // bf16 path: x packed into the same blocked layout [L0][H/64][Bp][64]
+    void* yb = nullptr;      // bf16 grid: ys packed [L1][H/64][Bp][64]
     float* c_all = nullptr;  // optional
     float* c_ring = nullptr; // workspace: fp32 cell-state ring
     int* flags = nullptr;    // workspace: readiness counters [ncells][MB]

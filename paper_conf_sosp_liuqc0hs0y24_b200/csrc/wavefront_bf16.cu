@@ -56,9 +56,14 @@ namespace ft {
 // libft.so): per CTA, cycles spent in each wait / work phase.
 enum TraceSlot {
     TR_P_FLAG = 0, TR_P_EMPTY, TR_M_FULL, TR_M_TEMPTY, TR_E_TFULL, TR_E_WORK, TR_E_CFLAG, TR_TOTAL,
-    TR_TILES, TR_SLOTS = 16
+    TR_TILES, TR_E_LDTM, TR_E_MATH, TR_E_STORE, TR_E_BAR, TR_E_REL, TR_SLOTS = 16
 };
 __device__ unsigned long long g_trace[1024 * TR_SLOTS];
+// per-tile event timestamps (%globaltimer, ns) of the leader CTA: 0 wait start, 1 deps ready,
+// 2 A loads issued, 3 MMA done (epilogue saw tfull), 4 counter released
+constexpr int EV_MAX_TILES = 65536;
+__device__ unsigned long long g_events[EV_MAX_TILES * 5];
+#define FT_EV(tile, k) do { if ((tile) < EV_MAX_TILES) g_events[(tile) * 5 + (k)] = globaltimer_ns(); } while (0)
 // register accumulators, flushed once per role (keeps the instrumented loops lean)
 #define FT_TR_ROLE unsigned long long _acc[TR_SLOTS] = {0}
 #define FT_TR_DECL long long _tr0 = 0
@@ -78,6 +83,7 @@ __device__ unsigned long long g_trace[1024 * TR_SLOTS];
 #define FT_TR_END(slot) ((void)0)
 #define FT_TR_ADD(slot, v) ((void)0)
 #define FT_TR_FLUSH(cond) ((void)0)
+#define FT_EV(tile, k) ((void)0)
 #endif
 
 namespace {
@@ -102,7 +108,7 @@ struct KCfg {
 #define FT_STAGES2 6
 #endif
     static constexpr int STAGES = CG == 1 ? 4 : FT_STAGES2;
-    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024;
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024 /* bias */ + 1024 /* align */;
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
 };
 
@@ -133,16 +139,35 @@ __device__ __forceinline__ Segment pick(const Segment (&seg)[3], int i) {
     return r;
 }
 
-// A operand K-chunk kc of segment sg for batch rows arow0 .. arow0+127: layer-0 inputs from the
-// caller's x / ys (3-D strided view), SSA activations from the blocked hb buffer (2-D, contiguous).
+// A operand K-chunk kc of segment sg for batch rows arow0 .. arow0+127, always from a blocked
+// [row][kc][Bp][64] buffer (2-D TMA, one contiguous 16 KiB box): the SSA activations hb, or the
+// layer-0 inputs x / ys packed into that layout at the start of the call (pack_rows_kernel).
 template <int CG>
 __device__ __forceinline__ void load_a(const Problem& P, const Maps& M, uint32_t dst, uint32_t bar,
                                        const Segment& sg, int kc, int arow0, bool fixed, uint64_t pol) {
-    if (fixed || sg.src != SRC_H) {
-        const CUtensorMap* am = (fixed || sg.src == SRC_X) ? &M.x : &M.ys;
-        tma_load_3d_hint_addr<CG>(dst, am, bar, fixed ? 0 : kc * BK, fixed ? 0 : sg.row, arow0, pol);
-    } else {
-        tma_load_2d_hint_addr<CG>(dst, &M.h, bar, 0, (int)hb_row(P, sg.row, kc, arow0), pol);
+    const CUtensorMap* am = (fixed || sg.src == SRC_X) ? &M.x : (sg.src == SRC_YS ? &M.ys : &M.h);
+    tma_load_2d_hint_addr<CG>(dst, am, bar, 0, fixed ? arow0 : (int)hb_row(P, sg.row, kc, arow0), pol);
+}
+
+// Pack a caller input [B][L][H] (batch-outermost, the ABI layout) into the blocked layout
+// [L][H/64][Bp][64] the A-operand boxes read; rows B..Bp-1 are zero.  One 16-byte vector per
+// thread-iteration, coalesced on the write side.
+__global__ void pack_rows_kernel(const __nv_bfloat16* __restrict__ src, __nv_bfloat16* __restrict__ dst,
+                                 int B, int L, int H, int Bp) {
+    const int KC = H / 64;
+    const long long nvec = (long long)L * KC * Bp * 8;
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < nvec;
+         v += (long long)gridDim.x * blockDim.x) {
+        const int j = (int)(v & 7);
+        long long r = v >> 3;
+        const int b = (int)(r % Bp);
+        r /= Bp;
+        const int kc = (int)(r % KC);
+        const int l = (int)(r / KC);
+        uint4 val = make_uint4(0, 0, 0, 0);
+        if (b < B)
+            val = __ldg(reinterpret_cast<const uint4*>(src + ((long long)b * L + l) * H + kc * 64 + j * 8));
+        reinterpret_cast<uint4*>(dst)[v] = val;
     }
 }
 
@@ -188,12 +213,14 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             long long prod[3];
             producers(P, tl.cell, prod);
             FT_TR_BEGIN();
+            if (rank == 0) FT_EV(tile, 0);
             if (!(P.debug & 1)) {
 #pragma unroll
                 for (int q = 0; q < 3; ++q)
                     if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
             }
             FT_TR_END(TR_P_FLAG);
+            if (rank == 0) FT_EV(tile, 1);
             fence_proxy_async_global();
         }
         int si = 0, kc = 0;
@@ -220,6 +247,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                 phase ^= 1;
             }
         }
+        if constexpr (!kWeights) if (rank == 0) FT_EV(tile, 2);
     }
     FT_TR_FLUSH(true);  // the two producers fill disjoint slots
 }
@@ -406,7 +434,8 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
 
 template <int CG>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
-                                             uint64_t* tfull, uint64_t* tempty, uint32_t rank) {
+                                             uint64_t* tfull, uint64_t* tempty, uint32_t rank,
+                                             float* sbias) {
     if (P.cell == CELL_LINEAR) {
         run_epilogue_linear<CG>(P, T, tmem_base, tfull, tempty, rank);
         return;
@@ -434,6 +463,14 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         const bool valid = b < P.B;
         const int n0 = tl.n * BNU + half * EPI_UNITS;
         FT_TR_DECL;
+        // (0) this tile's bias [4 gates][64 units] → shared memory while the MMAs still run (the
+        //     L1 is invalidated by every gpu-scope fence, so per-chunk global bias loads would
+        //     go to L2 on the epilogue's critical path)
+        {
+            const int e = threadIdx.x - 64;  // 0 .. 255
+            const int slice_b = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
+            sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + (e >> 6)) * P.H + tl.n * BNU + (e & 63));
+        }
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
         //     of the c-producer's counter, published to the other epilogue threads by bar.sync
         FT_TR_BEGIN();
@@ -460,25 +497,34 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         FT_TR_BEGIN();
         mbar_wait(&tfull[acc], acc_phase);
         if (leader_thread) FT_TR_END(TR_E_TFULL);
+        if (leader_thread && rank == 0) FT_EV(tile, 3);
         FT_TR_BEGIN();
         tc_fence_after();
 
         const int slice = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
-        const float* bias = T.b + (long long)slice * 4 * P.H;
         const bool top = (c.d == P.D - 1), last = is_last_pos(P, c);
         const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
                                (uint32_t)(half * EPI_UNITS);
         uint4 hp[EPI_UNITS / 8];
         float cv[EPI_UNITS];
+        const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
 #pragma unroll
         for (int u0 = 0; u0 < EPI_UNITS; u0 += 16) {
             __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
             float zi[16], zf[16], zo[16], zg[16];
+            long long _e0 = 0;
+#ifdef FT_TRACE
+            _e0 = clock64();
+#endif
             tmem_ld_32x32b_x16(tbase + 0 * BNU + u0, zi);
             tmem_ld_32x32b_x16(tbase + 1 * BNU + u0, zf);
             tmem_ld_32x32b_x16(tbase + 2 * BNU + u0, zo);
             tmem_ld_32x32b_x16(tbase + 3 * BNU + u0, zg);
             tmem_wait_ld();
+#ifdef FT_TRACE
+            if (leader_thread) _acc[TR_E_LDTM] += clock64() - _e0;
+            _e0 = clock64();
+#endif
             if (u0 + 16 == EPI_UNITS) {  // accumulator drained → hand it back to the MMA warp
                 tc_fence_before();
                 __syncwarp();
@@ -490,12 +536,19 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 }
             }
             if (P.debug & 2) continue;
-            const int n = n0 + u0;
+            const int ub = half * EPI_UNITS + u0;  // unit offset inside the tile
             float bi[16], bf[16], bo[16], bg[16];
-            load16(bias + 0 * P.H + n, bi);
-            load16(bias + 1 * P.H + n, bf);
-            load16(bias + 2 * P.H + n, bo);
-            load16(bias + 3 * P.H + n, bg);
+#pragma unroll
+            for (int v = 0; v < 16; v += 4) {
+                const float4 t0 = *reinterpret_cast<const float4*>(sbias + 0 * BNU + ub + v);
+                const float4 t1 = *reinterpret_cast<const float4*>(sbias + 1 * BNU + ub + v);
+                const float4 t2 = *reinterpret_cast<const float4*>(sbias + 2 * BNU + ub + v);
+                const float4 t3 = *reinterpret_cast<const float4*>(sbias + 3 * BNU + ub + v);
+                bi[v] = t0.x; bi[v + 1] = t0.y; bi[v + 2] = t0.z; bi[v + 3] = t0.w;
+                bf[v] = t1.x; bf[v + 1] = t1.y; bf[v + 2] = t1.z; bf[v + 3] = t1.w;
+                bo[v] = t2.x; bo[v + 1] = t2.y; bo[v + 2] = t2.z; bo[v + 3] = t2.w;
+                bg[v] = t3.x; bg[v + 1] = t3.y; bg[v + 2] = t3.z; bg[v + 3] = t3.w;
+            }
             float hv[16];
 #pragma unroll
             for (int v = 0; v < 16; ++v) {
@@ -513,25 +566,45 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                                             pack_bf16x2(hv[8 * w + 2], hv[8 * w + 3]),
                                             pack_bf16x2(hv[8 * w + 4], hv[8 * w + 5]),
                                             pack_bf16x2(hv[8 * w + 6], hv[8 * w + 7]));
+            // what downstream cells read — h (blocked SSA buffer hb) and c (ring) — stored per
+            // chunk so the stores overlap the next chunk's math
+            if (valid && !(P.debug & 2)) {
+                const int nn = n0 + u0;
+                uint4* hdst = reinterpret_cast<uint4*>(
+                    (__nv_bfloat16*)T.hb + hb_row(P, row_h, nn / 64, b) * 64 + (nn % 64));
+                __stcg(hdst + 0, hp[u0 / 8]);
+                __stcg(hdst + 1, hp[u0 / 8 + 1]);
+                float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn));
+#pragma unroll
+                for (int v = 0; v < 4; ++v)
+                    __stcg(cdst + v, make_float4(cv[u0 + 4 * v], cv[u0 + 4 * v + 1], cv[u0 + 4 * v + 2], cv[u0 + 4 * v + 3]));
+            }
+#ifdef FT_TRACE
+            if (leader_thread) _acc[TR_E_MATH] += clock64() - _e0;
+#endif
         }
-        // (2) what downstream cells read: h (blocked SSA buffer hb) and c (ring) → publish
+#ifdef FT_TRACE
+        long long _e1 = clock64();
+#endif
+        // (2) publish: every epilogue thread's h / c stores are ordered before the leader's
+        //     release by bar.sync (the release is cumulative)
         const long long hi = h_all_index(P, c, tl.axis, b, n0);
-        if (valid && !(P.debug & 2)) {
-            const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
-            uint4* hdst = reinterpret_cast<uint4*>(
-                (__nv_bfloat16*)T.hb + hb_row(P, row_h, n0 / 64, b) * 64 + (n0 % 64));
-#pragma unroll
-            for (int w = 0; w < EPI_UNITS / 8; ++w) __stcg(hdst + w, hp[w]);
-            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n0));
-#pragma unroll
-            for (int v = 0; v < EPI_UNITS / 4; ++v)
-                __stcg(cdst + v, make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]));
-        }
+#ifdef FT_TRACE
+        if (leader_thread) _acc[TR_E_STORE] += clock64() - _e1;
+        _e1 = clock64();
+#endif
         named_bar_sync(1, EPI_THREADS);
+#ifdef FT_TRACE
+        if (leader_thread) _acc[TR_E_BAR] += clock64() - _e1;
+        _e1 = clock64();
+#endif
         if (leader_thread) {
-            __threadfence();
             red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
             FT_TR_END(TR_E_WORK);
+            if (rank == 0) FT_EV(tile, 4);
+#ifdef FT_TRACE
+            _acc[TR_E_REL] += clock64() - _e1;
+#endif
         }
         // (3) outputs nobody inside the nest reads
         if (valid) {
@@ -584,6 +657,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     uint64_t* tfull = bars + 2 * C::STAGES;
     uint64_t* tempty = tfull + 2;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+    float* sbias = reinterpret_cast<float*>(smem + C::STAGES * C::STAGE_BYTES + 256);  // [4][64]
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const uint32_t rank = (CG == 2) ? cluster_ctarank() : 0u;
@@ -620,7 +694,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     } else if (warp == 10) {
         if (lane == 0) run_producer<CG, false>(P, T, M, sA, sB, full, empty, rank);
     } else {
-        run_epilogue<CG>(P, T, tmem_base, tfull, tempty, rank);
+        run_epilogue<CG>(P, T, tmem_base, tfull, tempty, rank, sbias);
     }
 
     tc_fence_before();
@@ -653,23 +727,6 @@ EncodeTiledFn get_encode_fn(std::string* err) {
     }
     fn = reinterpret_cast<EncodeTiledFn>(ptr);
     return fn;
-}
-
-// Activation view (hidden, rows, batch) with a (64, 1, 128) box, 128-byte swizzle.
-bool encode_act(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, long long rows,
-                int B, std::string* err) {
-    const cuuint64_t dims[3] = {(cuuint64_t)H, (cuuint64_t)rows, (cuuint64_t)B};
-    const cuuint64_t strides[2] = {(cuuint64_t)H * 2, (cuuint64_t)rows * H * 2};
-    const cuuint32_t box[3] = {(cuuint32_t)BK, 1, (cuuint32_t)ROWS};
-    const cuuint32_t es[3] = {1, 1, 1};
-    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides,
-                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                     CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-    if (r != CUDA_SUCCESS) {
-        if (err) *err = "cuTensorMapEncodeTiled(activation) failed: " + std::to_string((int)r);
-        return false;
-    }
-    return true;
 }
 
 // Blocked activation view (64 units, rows) with a (64, 128) box: one box = one contiguous 16 KiB
@@ -716,9 +773,10 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     if (!enc) return cudaErrorNotSupported;
     Maps M;
     const int slices = p.D * p.naxes;
-    if (!encode_act(enc, &M.x, t.x, p.H, p.L0, p.B, err)) return cudaErrorInvalidValue;
-    if (!encode_act(enc, &M.ys, p.kind == KIND_GRID ? t.ys : t.x, p.H,
-                    p.kind == KIND_GRID ? p.L1 : p.L0, p.B, err))
+    const int Bp = p.MB * p.BM;
+    if (!encode_blocked(enc, &M.x, t.xb, (long long)p.L0 * (p.H / 64) * Bp, err)) return cudaErrorInvalidValue;
+    if (!encode_blocked(enc, &M.ys, p.kind == KIND_GRID ? t.yb : t.xb,
+                        (long long)(p.kind == KIND_GRID ? p.L1 : p.L0) * (p.H / 64) * Bp, err))
         return cudaErrorInvalidValue;
     if (!encode_blocked(enc, &M.h, t.hb, hb_rows_total(p), err)) return cudaErrorInvalidValue;
     if (p.cell == CELL_LINEAR) {
@@ -751,6 +809,22 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     if (e != cudaSuccess) {
         if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
         return e;
+    }
+    // layer-0 inputs → blocked layout (part of the forward; ~T*H*Bp*4 bytes of traffic)
+    {
+        const long long nvec = (long long)p.L0 * (p.H / 64) * Bp * 8;
+        const int blocks = (int)((nvec + 255) / 256 < 4 * nsm ? (nvec + 255) / 256 : 4 * nsm);
+        pack_rows_kernel<<<blocks, 256, 0, s>>>((const __nv_bfloat16*)t.x, (__nv_bfloat16*)t.xb, p.B, p.L0, p.H, Bp);
+        if (p.kind == KIND_GRID) {
+            const long long nv2 = (long long)p.L1 * (p.H / 64) * Bp * 8;
+            const int b2 = (int)((nv2 + 255) / 256 < 4 * nsm ? (nv2 + 255) / 256 : 4 * nsm);
+            pack_rows_kernel<<<b2, 256, 0, s>>>((const __nv_bfloat16*)t.ys, (__nv_bfloat16*)t.yb, p.B, p.L1, p.H, Bp);
+        }
+        e = cudaGetLastError();
+        if (e != cudaSuccess) {
+            if (err) *err = std::string("input pack launch: ") + cudaGetErrorString(e);
+            return e;
+        }
     }
     cudaLaunchConfig_t cfg = {};
     cfg.blockDim = dim3(THREADS);
@@ -803,6 +877,12 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_trace(unsigned lo
         cudaMemcpyToSymbol(g_trace, zeros, sizeof(zeros));
     }
     return TR_SLOTS;
+}
+extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned long long* host, int ntiles) {
+    if (ntiles > EV_MAX_TILES) ntiles = EV_MAX_TILES;
+    cudaDeviceSynchronize();
+    if (cudaMemcpyFromSymbol(host, g_events, (size_t)ntiles * 5 * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    return ntiles;
 }
 #endif
 

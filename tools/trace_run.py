@@ -7,7 +7,7 @@ from paper_conf_sosp_liuqc0hs0y24_b200 import ft
 ft.LIB_PATH = os.path.abspath(os.environ.get("FT_TRACE_LIB", "build/trace/libft_trace.so"))
 L = ft.lib()
 L.ft_debug_trace.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int]
-NAMES = ["P_flag", "P_empty", "M_full", "M_tempty", "E_tfull", "E_work", "E_cflag", "total", "tiles"]
+NAMES = ["P_flag", "P_empty", "M_full", "M_tempty", "E_tfull", "E_work", "E_cflag", "total", "tiles", "E_ldtm", "E_math", "E_store", "E_bar", "E_rel"]
 for name in sys.argv[1:] or ["C3"]:
     if ":" in name:  # custom stacked spec  name:B,T,H,D
         B_, T_, H_, D_ = (int(v) for v in name.split(":")[1].split(","))
@@ -31,9 +31,9 @@ for name in sys.argv[1:] or ["C3"]:
     for _ in range(reps): fn()
     torch.cuda.synchronize()
     L.ft_debug_trace(buf, 1024 * 16, 1)
-    arr = np.array(buf[:], dtype=np.float64).reshape(1024, 16)[:148, :9] / reps
+    arr = np.array(buf[:], dtype=np.float64).reshape(1024, 16)[:148, :14] / reps
     tot = arr[:, 7].mean()
     print(name, "cycles/CTA/launch", f"{tot:.0f}", " tiles/CTA", arr[:, 8].mean())
-    for i, n in enumerate(NAMES[:7]):
+    for i, n in [(k, NAMES[k]) for k in list(range(7)) + list(range(9, 14))]:
         even = arr[0::2, i].mean() / tot * 100; odd = arr[1::2, i].mean() / tot * 100
         print(f"  {n:9s} leader {even:5.1f}%  peer {odd:5.1f}%   max {arr[:, i].max()/tot*100:5.1f}%")
