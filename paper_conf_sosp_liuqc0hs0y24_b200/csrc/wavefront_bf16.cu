@@ -329,18 +329,6 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
     return *reinterpret_cast<uint32_t*>(&v);
 }
 
-__device__ __forceinline__ void load16(const float* src, float (&v)[16]) {
-    const float4* s4 = reinterpret_cast<const float4*>(src);
-#pragma unroll
-    for (int q = 0; q < 4; ++q) {
-        const float4 t = __ldg(s4 + q);
-        v[4 * q + 0] = t.x;
-        v[4 * q + 1] = t.y;
-        v[4 * q + 2] = t.z;
-        v[4 * q + 3] = t.w;
-    }
-}
-
 // 8 epilogue warps: warp w reads TMEM lane quadrant w % 4 (rows) and unit half (w - 2) / 4
 // (32 of the tile's 64 units); one thread per batch row.
 constexpr int EPI_WARPS = 8;
@@ -501,7 +489,6 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         FT_TR_BEGIN();
         tc_fence_after();
 
-        const int slice = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
         const bool top = (c.d == P.D - 1), last = is_last_pos(P, c);
         const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
                                (uint32_t)(half * EPI_UNITS);

@@ -14,6 +14,8 @@ def timeit(fn, reps=10, warm=3):
         s.record(); fn(); e.record(); torch.cuda.synchronize(); ts.append(s.elapsed_time(e))
     return float(np.median(ts)), float(np.min(ts))
 
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)) + "/..")
+import bench
 res = {}
 for name in sys.argv[1:] or ["C2", "C3", "C4", "C5"]:
     if ":" in name:  # custom stacked spec  name:B,T,H,D
@@ -37,6 +39,10 @@ for name in sys.argv[1:] or ["C2", "C3", "C4", "C5"]:
             flops = sum(2*B*4*H*(H*T + H*max(0, T-s)) for s in dil)
         else:
             flops = 16 * H * H * T * D * B
+    cs = bench.ClockSampler(0)
+    cs.start()
     med, mn = timeit(fn, reps=int(os.environ.get("QT_REPS", "10")), warm=int(os.environ.get("QT_WARM", "3")))
-    res[name] = dict(ms_median=med, ms_min=mn, tflops=flops / med / 1e9, seq_per_s=c["batch"] / med * 1e3)
+    clk = cs.stop()
+    res[name] = dict(ms_median=med, ms_min=mn, tflops=flops / med / 1e9, seq_per_s=c["batch"] / med * 1e3,
+                     sm_mhz=(clk or {}).get("sm_mhz"), power_w=(clk or {}).get("power_w_median"))
     print(name, json.dumps(res[name]), flush=True)
