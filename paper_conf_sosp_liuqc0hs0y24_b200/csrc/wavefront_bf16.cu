@@ -91,25 +91,28 @@ namespace {
 using namespace sm100;
 
 constexpr int ROWS = BF16_BM;  // 128 batch rows per CTA = TMEM lanes
-constexpr int BNU = BF16_BNU;  // 64 hidden units per tile
-constexpr int BN = 4 * BNU;    // 256 = UMMA N (i | f | o | ĝ)
-constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16
+constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16 (A operand)
 constexpr int UK = 16;         // UMMA K for kind::f16
 constexpr int THREADS = 352;  // warp 0 weight TMA, 1 MMA, 2-9 epilogue, 10 activation TMA
-constexpr int TMEM_COLS = 2 * BN;  // double-buffered accumulator
 
-template <int CG>
+// Tile configuration: CG CTAs per tile (1 or a cta_group::2 pair), U hidden units per N-tile
+// (64: N = 256 with 128-byte-swizzled weight atoms; 32: N = 128 with 64-byte swizzle — twice the
+// tiles per diagonal at half the per-tile latency, for diagonals too narrow to fill the GPU).
+template <int CG, int U>
 struct KCfg {
-    static constexpr int GATES = 4 / CG;                       // weight gate boxes per CTA
+    static constexpr int BNU = U;
+    static constexpr int BN = 4 * U;                           // UMMA N (i | f | o | ĝ)
+    static constexpr int TMEM_COLS = 2 * BN;                   // double-buffered accumulator
+    static constexpr int GATES = 4 / CG;                       // weight gate atoms per CTA
+    static constexpr int WROW = U * 2;                         // bytes per weight smem row
+    static constexpr uint32_t WLAYOUT = U == 64 ? 2u : 4u;     // SWIZZLE_128B / SWIZZLE_64B
     static constexpr int A_BYTES = ROWS * BK * 2;              // 16 KiB
-    static constexpr int B_BYTES = GATES * BNU * BK * 2;       // 32 KiB (CG 1) / 16 KiB (CG 2)
+    static constexpr int B_BYTES = GATES * U * BK * 2;         // weight atoms of one K chunk
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-#ifndef FT_STAGES2
-#define FT_STAGES2 6
-#endif
-    static constexpr int STAGES = CG == 1 ? 4 : FT_STAGES2;
+    static constexpr int STAGES = (196 * 1024) / STAGE_BYTES;  // 4 / 6 / 6 / 8
     static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024 /* bias */ + 1024 /* align */;
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
+    static constexpr int EPI_UNITS = U / 2;                    // units per epilogue thread
 };
 
 struct Maps {
@@ -177,11 +180,11 @@ __global__ void pack_rows_kernel(const __nv_bfloat16* __restrict__ src, __nv_bfl
 // full barrier (in the leader CTA) takes one expect-tx arrival from each of the leader's two
 // producers; the peer CTA's producers only issue loads.  Splitting halves the serial TMA issue
 // work per thread (the role trace showed one thread issuing both was the limiter).
-template <int CG, bool kWeights>
+template <int CG, int U, bool kWeights>
 __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
                                              uint8_t* sA, uint8_t* sB, uint64_t* full,
                                              uint64_t* empty, uint32_t rank) {
-    using C = KCfg<CG>;
+    using C = KCfg<CG, U>;
     const uint32_t sA0 = smem_u32(sA), sB0 = smem_u32(sB);
     const uint32_t full0 = (CG == 2) ? mapa_shared(smem_u32(full), 0) : smem_u32(full);
     int stage = 0;
@@ -203,7 +206,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         const int nchunks = ns * kchunks;
         const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
         const bool lin = P.cell == CELL_LINEAR;
-        const int bn = (fixed || lin) ? 0 : tl.n * BNU;
+        const int bn = (fixed || lin) ? 0 : tl.n * U;
         const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
         FT_TR_DECL;
         if constexpr (!kWeights) {
@@ -253,11 +256,11 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
 }
 
 // ------------------------------------------------------------------------------ MMA issuer
-template <int CG>
+template <int CG, int U>
 __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, uint8_t* sA,
                                         uint8_t* sB, uint64_t* full, uint64_t* empty,
                                         uint64_t* tfull, uint64_t* tempty) {
-    using C = KCfg<CG>;
+    using C = KCfg<CG, U>;
     int stage = 0;
     uint32_t phase = 0;
     int acc = 0;
@@ -265,10 +268,10 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
     Cursor cur = cursor_begin();
     const int kchunks = P.H / BK;
     // A: K-major, SW128: 128-B rows, 8-row groups 1024 B apart (SBO); K step = +32 B.
-    // B: MN-major, SW128: 64-n atoms (one per gate) 8 KiB apart (LBO), 8-k groups 1024 B apart
-    //    (SBO); K step of 16 rows = +2048 B.  CG 2: each CTA holds half the gate atoms.
+    // B: MN-major, U-unit swizzle atoms (one per gate) U*64*2 B apart (LBO), 8-k-row groups
+    //    8*WROW apart (SBO); K step of 16 rows = 16*WROW.  CG 2: each CTA holds half the atoms.
     const uint64_t adesc0 = make_sdesc(smem_u32(sA), 16, 1024);
-    const uint64_t bdesc0 = make_sdesc(smem_u32(sB), 8192, 1024);
+    const uint64_t bdesc0 = make_sdesc(smem_u32(sB), U * BK * 2, 8 * C::WROW, C::WLAYOUT);
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
     FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
@@ -280,7 +283,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         FT_TR_END(TR_M_TEMPTY);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+        const uint32_t d_tmem = tmem_base + (uint32_t)(acc * C::BN);
         for (int c = 0; c < nchunks; ++c) {
             FT_TR_BEGIN();
             mbar_wait(&full[stage], phase);
@@ -299,7 +302,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
 #pragma unroll
             for (int kk = 0; kk < BK / UK; ++kk)
                 umma_f16_cg<CG>(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
-                                bd + (uint64_t)((kk * UK * 128) >> 4), C::IDESC, (c | kk) != 0);
+                                bd + (uint64_t)((kk * UK * C::WROW) >> 4), C::IDESC, (c | kk) != 0);
             umma_commit_cg<CG>(&empty[stage]);
             }
             if (++stage == C::STAGES) {
@@ -333,14 +336,14 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
 // (32 of the tile's 64 units); one thread per batch row.
 constexpr int EPI_WARPS = 8;
 constexpr int EPI_THREADS = EPI_WARPS * 32;
-constexpr int EPI_UNITS = BNU / 2;  // units per thread
 
 // Listing 1's linear cell: y = z + s, s = the previous step's output (fp32 ring), 0 at t = 0.
 // The 256 accumulator columns are 256 consecutive units; warp half h takes columns h*128 ...
-template <int CG>
+template <int CG, int U>
 __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tensors& T,
                                                     uint32_t tmem_base, uint64_t* tfull,
                                                     uint64_t* tempty, uint32_t rank) {
+    using C = KCfg<CG, U>;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3, half = (warp - 2) >> 2, row = q * 32 + lane;
     const bool leader_thread = (threadIdx.x == 64);
@@ -357,22 +360,22 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
         const long long cprod = c_producer(P, tl, &ci, &cj);
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
-        const int n0 = tl.n * 4 * BNU + half * 2 * BNU;
+        const int n0 = tl.n * 4 * C::BNU + half * 2 * C::BNU;
         if (cprod >= 0 && leader_thread)
             wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
         named_bar_sync(1, EPI_THREADS);
         mbar_wait(&tfull[acc], acc_phase);
         tc_fence_after();
-        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
-                               (uint32_t)(half * 2 * BNU);
+        const uint32_t tbase = tmem_base + (uint32_t)(acc * C::BN) + ((uint32_t)(q * 32) << 16) +
+                               (uint32_t)(half * 2 * C::BNU);
         const int row_h = h_row(P, c.d, c.i, c.j, 0);
 #pragma unroll 1
-        for (int u0 = 0; u0 < 2 * BNU; u0 += 16) {
+        for (int u0 = 0; u0 < 2 * C::BNU; u0 += 16) {
             __syncwarp();
             float z[16];
             tmem_ld_32x32b_x16(tbase + u0, z);
             tmem_wait_ld();
-            if (u0 + 16 == 2 * BNU) {
+            if (u0 + 16 == 2 * C::BNU) {
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) {
@@ -420,13 +423,17 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
     }
 }
 
-template <int CG>
+template <int CG, int U>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
                                              uint64_t* tfull, uint64_t* tempty, uint32_t rank,
                                              float* sbias) {
-    if (P.cell == CELL_LINEAR) {
-        run_epilogue_linear<CG>(P, T, tmem_base, tfull, tempty, rank);
-        return;
+    using C = KCfg<CG, U>;
+    constexpr int EPI_UNITS = C::EPI_UNITS;
+    if constexpr (U == 64) {
+        if (P.cell == CELL_LINEAR) {
+            run_epilogue_linear<CG, U>(P, T, tmem_base, tfull, tempty, rank);
+            return;
+        }
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3;                 // TMEM lane quadrant this warp may access
@@ -449,7 +456,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         const long long cprod = c_producer(P, tl, &ci, &cj);
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
-        const int n0 = tl.n * BNU + half * EPI_UNITS;
+        const int n0 = tl.n * U + half * EPI_UNITS;
         FT_TR_DECL;
         // (0) this tile's bias [4 gates][64 units] → shared memory while the MMAs still run (the
         //     L1 is invalidated by every gpu-scope fence, so per-chunk global bias loads would
@@ -457,7 +464,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         {
             const int e = threadIdx.x - 64;  // 0 .. 255
             const int slice_b = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
-            sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + (e >> 6)) * P.H + tl.n * BNU + (e & 63));
+            if (e < 4 * U) sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + e / U) * P.H + tl.n * U + e % U);
         }
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
         //     of the c-producer's counter, published to the other epilogue threads by bar.sync
@@ -490,7 +497,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         tc_fence_after();
 
         const bool top = (c.d == P.D - 1), last = is_last_pos(P, c);
-        const uint32_t tbase = tmem_base + (uint32_t)(acc * BN) + ((uint32_t)(q * 32) << 16) +
+        const uint32_t tbase = tmem_base + (uint32_t)(acc * C::BN) + ((uint32_t)(q * 32) << 16) +
                                (uint32_t)(half * EPI_UNITS);
         uint4 hp[EPI_UNITS / 8];
         float cv[EPI_UNITS];
@@ -503,10 +510,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #ifdef FT_TRACE
             _e0 = clock64();
 #endif
-            tmem_ld_32x32b_x16(tbase + 0 * BNU + u0, zi);
-            tmem_ld_32x32b_x16(tbase + 1 * BNU + u0, zf);
-            tmem_ld_32x32b_x16(tbase + 2 * BNU + u0, zo);
-            tmem_ld_32x32b_x16(tbase + 3 * BNU + u0, zg);
+            tmem_ld_32x32b_x16(tbase + 0 * U + u0, zi);
+            tmem_ld_32x32b_x16(tbase + 1 * U + u0, zf);
+            tmem_ld_32x32b_x16(tbase + 2 * U + u0, zo);
+            tmem_ld_32x32b_x16(tbase + 3 * U + u0, zg);
             tmem_wait_ld();
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_LDTM] += clock64() - _e0;
@@ -527,10 +534,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             float bi[16], bf[16], bo[16], bg[16];
 #pragma unroll
             for (int v = 0; v < 16; v += 4) {
-                const float4 t0 = *reinterpret_cast<const float4*>(sbias + 0 * BNU + ub + v);
-                const float4 t1 = *reinterpret_cast<const float4*>(sbias + 1 * BNU + ub + v);
-                const float4 t2 = *reinterpret_cast<const float4*>(sbias + 2 * BNU + ub + v);
-                const float4 t3 = *reinterpret_cast<const float4*>(sbias + 3 * BNU + ub + v);
+                const float4 t0 = *reinterpret_cast<const float4*>(sbias + 0 * U + ub + v);
+                const float4 t1 = *reinterpret_cast<const float4*>(sbias + 1 * U + ub + v);
+                const float4 t2 = *reinterpret_cast<const float4*>(sbias + 2 * U + ub + v);
+                const float4 t3 = *reinterpret_cast<const float4*>(sbias + 3 * U + ub + v);
                 bi[v] = t0.x; bi[v + 1] = t0.y; bi[v + 2] = t0.z; bi[v + 3] = t0.w;
                 bf[v] = t1.x; bf[v + 1] = t1.y; bf[v + 2] = t1.z; bf[v + 3] = t1.w;
                 bo[v] = t2.x; bo[v + 1] = t2.y; bo[v + 2] = t2.z; bo[v + 3] = t2.w;
@@ -628,11 +635,11 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     FT_TR_FLUSH(leader_thread);
 }
 
-template <int CG>
+template <int CG, int U>
 __global__ void __launch_bounds__(THREADS, 1)
 wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
                       const __grid_constant__ Maps M) {
-    using C = KCfg<CG>;
+    using C = KCfg<CG, U>;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     uint8_t* smem = smem_raw + pad;
@@ -667,7 +674,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         tma_prefetch_desc(&M.W);
         tma_prefetch_desc(&M.U);
     }
-    if (warp == 1) tmem_alloc_cg<CG>(tmem_slot, TMEM_COLS);
+    if (warp == 1) tmem_alloc_cg<CG>(tmem_slot, C::TMEM_COLS);
     tc_fence_before();
     __syncthreads();
     if constexpr (CG == 2) cluster_sync();
@@ -675,13 +682,13 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == 0) {
-        if (lane == 0) run_producer<CG, true>(P, T, M, sA, sB, full, empty, rank);
+        if (lane == 0) run_producer<CG, U, true>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
-        if (lane == 0 && rank == 0) run_mma<CG>(P, tmem_base, sA, sB, full, empty, tfull, tempty);
+        if (lane == 0 && rank == 0) run_mma<CG, U>(P, tmem_base, sA, sB, full, empty, tfull, tempty);
     } else if (warp == 10) {
-        if (lane == 0) run_producer<CG, false>(P, T, M, sA, sB, full, empty, rank);
+        if (lane == 0) run_producer<CG, U, false>(P, T, M, sA, sB, full, empty, rank);
     } else {
-        run_epilogue<CG>(P, T, tmem_base, tfull, tempty, rank, sbias);
+        run_epilogue<CG, U>(P, T, tmem_base, tfull, tempty, rank, sbias);
     }
 
     tc_fence_before();
@@ -689,7 +696,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     if constexpr (CG == 2) cluster_sync();
     if (warp == 1) {
         tc_fence_after();
-        tmem_dealloc_cg<CG>(tmem_base, TMEM_COLS);
+        tmem_dealloc_cg<CG>(tmem_base, C::TMEM_COLS);
     }
     if (threadIdx.x == 0) FT_TR_END(TR_TOTAL);
     FT_TR_FLUSH(threadIdx.x == 0);
@@ -737,14 +744,15 @@ bool encode_blocked(EncodeTiledFn enc, CUtensorMap* m, const void* base, long lo
 // Weight view (n, k, gate, slice) with a (64, 64, gates, 1) box, 128-byte swizzle: the box is
 // the [i | f | o | ĝ] (CG 1) or [i | f] / [o | ĝ] (CG 2) x 64-unit slab of one 64-row K chunk.
 bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int krows, int slices,
-               int gates, std::string* err) {
+               int gates, int units, std::string* err) {
     const cuuint64_t dims[4] = {(cuuint64_t)H, (cuuint64_t)krows, 4, (cuuint64_t)slices};
     const cuuint64_t strides[3] = {(cuuint64_t)H * 2, (cuuint64_t)krows * H * 2,
                                    (cuuint64_t)4 * krows * H * 2};
-    const cuuint32_t box[4] = {(cuuint32_t)BNU, (cuuint32_t)BK, (cuuint32_t)gates, 1};
+    const cuuint32_t box[4] = {(cuuint32_t)units, (cuuint32_t)BK, (cuuint32_t)gates, 1};
     const cuuint32_t es[4] = {1, 1, 1, 1};
     CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides,
-                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                     box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                     units == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
                      CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS) {
         if (err) *err = "cuTensorMapEncodeTiled(weight) failed: " + std::to_string((int)r);
@@ -753,9 +761,9 @@ bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int k
     return true;
 }
 
-template <int CG>
+template <int CG, int U>
 cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
-    using C = KCfg<CG>;
+    using C = KCfg<CG, U>;
     EncodeTiledFn enc = get_encode_fn(err);
     if (!enc) return cudaErrorNotSupported;
     Maps M;
@@ -782,8 +790,8 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         }
         M.U = M.W;
     } else {
-        if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, err)) return cudaErrorInvalidValue;
-        if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, err))
+        if (!encode_wt(enc, &M.W, t.W, p.H, p.H, slices, C::GATES, U, err)) return cudaErrorInvalidValue;
+        if (!encode_wt(enc, &M.U, t.U, p.H, u_krows(p), slices, C::GATES, U, err))
             return cudaErrorInvalidValue;
     }
 
@@ -791,7 +799,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     cudaError_t e = cudaGetDevice(&dev);
     if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG>,
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
     if (e != cudaSuccess) {
         if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
@@ -835,7 +843,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         cfg.attrs = attr;
         cfg.numAttrs = 1;
         int nclusters = 0;
-        e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG>, &cfg);
+        e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U>, &cfg);
         if (e != cudaSuccess || nclusters < 1) {
             if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
             return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
@@ -846,7 +854,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     cfg.gridDim = dim3((unsigned)grid);
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG>, p, t, M);
+    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, p, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
 }
@@ -885,7 +893,35 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
             if (bnu) return launch_wavefront_resident(p, t, s, bnu, err);
         }
     }
-    return p.BM == 2 * ROWS ? launch_cg<2>(p, t, s, err) : launch_cg<1>(p, t, s, err);
+    // N-tile width: 64 units by default; 32 units when a diagonal at 64 units cannot give every
+    // CTA group a tile (few cells per diagonal, e.g. the 6-layer dilated C4): twice the tiles, half
+    // the per-tile latency on the dependency chain.
+    const int cg = p.BM == 2 * ROWS ? 2 : 1;
+    int dev = 0, nsm = 148;
+    if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    long long max_cells = 0;
+    if (p.kind == KIND_SEQ) {
+        max_cells = p.D < p.L0 ? p.D : p.L0;
+    } else {
+        for (int k = 0; k < p.D + p.L0 + p.L1 - 2; ++k) {
+            long long n = 0;
+            for (int d = 0; d < p.D && d <= k; ++d) {
+                const int r = k - d;
+                const int ilo = r - (p.L1 - 1) > 0 ? r - (p.L1 - 1) : 0, ihi = r < p.L0 - 1 ? r : p.L0 - 1;
+                if (ihi >= ilo) n += ihi - ilo + 1;
+            }
+            if (n > max_cells) max_cells = n;
+        }
+    }
+    int units = (max_cells * p.naxes * p.MB * p.NT < nsm / cg && p.cell == CELL_LSTM && p.H % 32 == 0) ? 32 : 64;
+    if (const char* env = getenv("FT_TILE_UNITS")) units = atoi(env) == 32 && p.cell == CELL_LSTM ? 32 : 64;
+    if (units == 64)
+        return cg == 2 ? launch_cg<2, 64>(p, t, s, err) : launch_cg<1, 64>(p, t, s, err);
+    Problem q = p;
+    q.BNU = 32;
+    q.NT = p.H / 32;
+    q.ntiles = q.ncells * q.naxes * q.MB * q.NT;
+    return cg == 2 ? launch_cg<2, 32>(q, t, s, err) : launch_cg<1, 32>(q, t, s, err);
 }
 
 }  // namespace ft

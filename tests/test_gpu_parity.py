@@ -227,3 +227,26 @@ def test_bf16_linear_rnn(B, T, H, D):
     ys = ft.stacked_rnn(dev(p["x"], torch.bfloat16), dev(p["W"], torch.bfloat16))
     torch.cuda.synchronize()
     _check({"ys": ys}, {"ys": oracle.stacked_rnn(p["x"], p["W"])}, torch.bfloat16, ("ys",), ctx="bf16 linear")
+
+
+# ------------------------------------------------------------------------- 32-unit N tiles
+@pytest.mark.parametrize("B,T,H,D,dil", [(130, 4, 128, 3, None), (64, 5, 192, 2, None),
+                                         (256, 9, 256, 3, [1, 2, 4]), (20, 13, 128, 3, [3, 1, 7])])
+def test_bf16_narrow_tiles(B, T, H, D, dil, monkeypatch):
+    """The streaming kernel with 32-unit N tiles (N = 128, 64-byte-swizzled weight atoms), chosen
+    automatically for narrow diagonals (C4) — forced here, streaming (not weight-resident)."""
+    monkeypatch.setenv("FT_TILE_UNITS", "32")
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    p = ftgen.stacked_inputs(B, T, H, D, 1111 + B, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"u32 {B,T,H,D,dil}")
+
+
+def test_bf16_narrow_tiles_grid(monkeypatch):
+    monkeypatch.setenv("FT_TILE_UNITS", "32")
+    g = ftgen.grid_inputs(130, 3, 2, 128, 2, 1212, "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx="u32 grid")

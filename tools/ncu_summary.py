@@ -69,6 +69,9 @@ def main():
     os.makedirs("profiles", exist_ok=True)
     with open(f"profiles/{tag}_ncu_summary.json", "w") as f:
         json.dump(summ, f, indent=1)
+    if launches == "-":
+        print(json.dumps(summ, indent=1))
+        return
     # launch list: kernel name, count, mean duration, share
     rows = list(csv.reader(open(launches)))
     start = next(i for i, r in enumerate(rows) if r and r[0] == "ID")
