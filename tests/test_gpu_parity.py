@@ -250,3 +250,47 @@ def test_bf16_narrow_tiles_grid(monkeypatch):
     torch.cuda.synchronize()
     ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
     _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx="u32 grid")
+
+
+# ------------------------------------------------------------------------- more edge cases
+@pytest.mark.parametrize("B,T,H,D", [(1, 7, 128, 3), (256, 1, 128, 4), (5, 3, 64, 32)])
+def test_bf16_streaming_edges(B, T, H, D, monkeypatch):
+    """Streaming kernel edges: one batch row, one time step (only boundary cells), and the
+    paper's depth 32 (Table 6) with its 34-diagonal wavefront."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    p = ftgen.stacked_inputs(B, T, H, D, 1313 + D, "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"edge {B,T,H,D}")
+
+
+def test_bf16_dilation_at_least_T():
+    """Layers whose dilation ≥ T never read a recurrent state (P7c on the GPU path)."""
+    p = ftgen.stacked_inputs(6, 5, 64, 3, 1414, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=[1, 5, 9], want_all=True)
+    _check(got, _oracle_stacked(p, dil=[1, 5, 9], want_all=True), torch.bfloat16, ALL, ctx="dil>=T")
+
+
+@pytest.mark.parametrize("Lx,Ly", [(5, 1), (1, 4)])
+def test_bf16_grid_one_axis(Lx, Ly):
+    """Grid with one axis of length 1 (the P8 reduction case) on the tcgen05 path."""
+    g = ftgen.grid_inputs(7, Lx, Ly, 64, 3, 1515 + Lx, "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx=f"grid {Lx}x{Ly}")
+
+
+def test_bf16_workspace_reuse_and_stream():
+    """One workspace reused across different problems on a non-default stream: every call
+    re-initialises its counters (no state leaks between calls)."""
+    ws = ft.Workspace()
+    s = torch.cuda.Stream()
+    for (B, T, H, D) in [(130, 4, 128, 2), (40, 6, 64, 3), (130, 4, 128, 2)]:
+        p = ftgen.stacked_inputs(B, T, H, D, 1616 + B + T, "bf16")
+        with torch.cuda.stream(s):
+            x, W, U = (dev(p[k], torch.bfloat16) for k in ("x", "W", "U"))
+            b = dev(p["b"], torch.float32)
+            r = ft.stacked_lstm(x, W, U, b, workspace=ws, stream=s)
+        s.synchronize()
+        _check(r, _oracle_stacked(p), torch.bfloat16, OUT, ctx=f"reuse {B,T,H,D}")
