@@ -313,6 +313,16 @@ def run_ours(args):
                 "note": "launch duration = one ft_stacked_lstm_fwd call: counter reset + x pack "
                         "(52 MB) + the persistent wavefront kernel, CUDA events on the launch stream"}
 
+    # the same achieved rate against the tensor peak at the clock the run actually had (148 SMs x
+    # 8192 dense bf16 FLOP/clk/SM x the median SM clock sampled during the timed region): the
+    # kernel's efficiency with the power cap's clock taken out
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    if clocks and clocks.get("sm_mhz"):
+        clk_peak = nsm * 8192 * clocks["sm_mhz"] * 1e6 / 1e12
+        roofline["clock_normalized"] = {"peak_at_sampled_clock_tflops": clk_peak,
+                                        "frac": achieved / clk_peak,
+                                        "sm_mhz": clocks["sm_mhz"]}
+
     # end to end through the public host-buffer C-ABI call (pinned host in/out, copies timed)
     e2e = None
     if True:  # every rank: its own shard through the host-buffer call; max over ranks below
