@@ -80,6 +80,10 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
     p->NT = (H + p->BNU - 1) / p->BNU;
     p->ncells = (long long)D * L0 * L1;
     p->ntiles = p->ncells * p->naxes * p->MB * p->NT;
+    // bf16: TMA row coordinates into the blocked buffers are int32
+    if (dt == FT_BF16 && (ft::hb_rows_total(*p) >= (1ll << 31) ||
+                          (long long)L0 * (H / 64) * p->MB * p->BM >= (1ll << 31)))
+        return fail(FT_ERR_UNSUPPORTED, "problem too large: blocked activation rows exceed int32 TMA coordinates");
     if (kind == ft::KIND_SEQ) {
         int off = 0;
         for (int d = 0; d < D; ++d) {

@@ -39,7 +39,9 @@ struct Problem {
     int flag_mult;       // counter increments per tile (CTAs per tile: 2 for a tcgen05 CTA pair)
     int resident_layers; // bf16: layers whose weights are kept in L2 (evict_last); others stream
     int debug;           // timing experiments only (env FT_DEBUG; results invalid when != 0):
-                         // bit 0 skip dependency waits, bit 1 skip the epilogue math/stores
+                         // bit 0 skip dependency waits, bit 1 skip the epilogue math/stores;
+                         // bit 6 (64) = stress mode: random delays before each counter release
+                         // (results stay valid; used by tests to shake out ordering bugs)
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT
     int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)

@@ -593,6 +593,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         _e1 = clock64();
 #endif
         if (leader_thread) {
+            if (P.debug & 64) {  // stress mode (tests): a pseudo-random delay before publishing
+                const uint32_t h = (uint32_t)(tile * 2654435761u) ^ (uint32_t)blockIdx.x * 40503u;
+                __nanosleep(200 + (h & 4095u));
+            }
             red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
             FT_TR_END(TR_E_WORK);
             if (rank == 0) FT_EV(tile, 4);

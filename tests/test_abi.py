@@ -64,6 +64,7 @@ def _call(**over):
     (dict(h_all=FAKE + 4), ft.FT_ERR_INVALID_ARGUMENT),
     (dict(hidden=96), ft.FT_ERR_UNSUPPORTED),
     (dict(depth=65), ft.FT_ERR_UNSUPPORTED),
+    (dict(depth=64, seq=20000, hidden=4096, batch=256), ft.FT_ERR_UNSUPPORTED),  # int32 TMA rows
     (dict(workspace_bytes=16), ft.FT_ERR_WORKSPACE_TOO_SMALL),
     (dict(workspace=None, workspace_bytes=0), ft.FT_ERR_INVALID_ARGUMENT),
 ])

@@ -294,3 +294,42 @@ def test_bf16_workspace_reuse_and_stream():
             r = ft.stacked_lstm(x, W, U, b, workspace=ws, stream=s)
         s.synchronize()
         _check(r, _oracle_stacked(p), torch.bfloat16, OUT, ctx=f"reuse {B,T,H,D}")
+
+
+# ------------------------------------------------------------------------- robustness
+@pytest.mark.parametrize("B,T,H,D,dil", [(130, 6, 128, 3, None), (256, 5, 64, 4, [1, 2, 3, 1])])
+def test_bf16_stress_delayed_release(B, T, H, D, dil, monkeypatch):
+    """Stress mode (FT_DEBUG=64): a pseudo-random delay before every counter release reorders
+    completions across CTAs; results must not change (shakes out missing acquire/release or
+    proxy fences — SURVEY T6)."""
+    monkeypatch.setenv("FT_DEBUG", "64")
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    p = ftgen.stacked_inputs(B, T, H, D, 1717 + B, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx="stress")
+
+
+def test_bf16_cuda_graph_capture_replay():
+    """The forward (counter reset + input pack + persistent kernel) captures into a CUDA graph
+    and replays with new inputs copied into the captured buffers (the serving path)."""
+    B, T, H, D = 130, 5, 128, 3
+    p1 = ftgen.stacked_inputs(B, T, H, D, 1818, "bf16")
+    p2 = ftgen.stacked_inputs(B, T, H, D, 1819, "bf16")
+    x, W, U = (dev(p1[k], torch.bfloat16) for k in ("x", "W", "U"))
+    b = dev(p1["b"], torch.float32)
+    ws = ft.Workspace()
+    s = torch.cuda.Stream()
+    out = {"y": torch.empty((B, T, H), dtype=torch.bfloat16, device="cuda"),
+           "h_n": torch.empty((B, D, H), dtype=torch.bfloat16, device="cuda"),
+           "c_n": torch.empty((B, D, H), dtype=torch.float32, device="cuda")}
+    with torch.cuda.stream(s):
+        ft.stacked_lstm(x, W, U, b, workspace=ws, out=out, stream=s)  # warm-up (sizes workspace)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        ft.stacked_lstm(x, W, U, b, workspace=ws, out=out, stream=s)
+    x.copy_(dev(p2["x"], torch.bfloat16))
+    g.replay()
+    torch.cuda.synchronize()
+    ref = oracle.stacked_lstm(p2["x"], p1["W"], p1["U"], p1["b"])
+    _check(out, ref, torch.bfloat16, OUT, ctx="graph")
