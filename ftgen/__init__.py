@@ -96,6 +96,16 @@ def linear_rnn_inputs(batch, seq, hidden, depth, seed, dtype="bf16", scale=1.0):
     )
 
 
+def b2b_inputs(M, N, K, P, seed, dtype="bf16"):
+    """Inputs of ft_b2b_gemm_fwd: A [M][K] ~ U(-1,1), B [K][N] ~ U(±1/√K), C [N][P] ~ U(±1/√N)
+    (scaled so S = A@B and D = S@C stay O(1))."""
+    return dict(
+        A=_draw(seed, S_X, (M, K), 1.0, dtype),
+        B=_draw(seed, S_W, (K, N), 1.0 / np.sqrt(K), dtype),
+        C=_draw(seed, S_U, (N, P), 1.0 / np.sqrt(N), dtype),
+    )
+
+
 def grid_inputs(batch, len_x, len_y, hidden, depth, seed, dtype="bf16", scale=1.0):
     """Inputs of ft_grid_rnn_fwd: x [B][Lx][H], ys [B][Ly][H], W [D][2][4][H][H],
     U [D][2][4][2H][H], b [D][2][4][H]."""

@@ -42,7 +42,8 @@ def lib():
         build()
         _lib = ctypes.CDLL(LIB_PATH)
         for sfx in ("f64", "f32"):
-            for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell", "stacked_rnn"):
+            for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell", "stacked_rnn",
+                         "b2b_gemm"):
                 fn = getattr(_lib, f"ft_oracle_{name}_{sfx}")
                 fn.restype = ctypes.c_int if name != "lstm_cell" else None
     return _lib
@@ -168,3 +169,18 @@ def stacked_rnn(x, W, precision="f64"):
     if rc:
         raise RuntimeError(f"oracle stacked_rnn failed: {rc}")
     return ys
+
+
+def b2b_gemm(A, B, C, precision="f64"):
+    """Back-to-back GEMMs (Table 6; reading R22): D = (A @ B) @ C.
+    A [M][K], B [K][N], C [N][P] → D [M][P]."""
+    dt = _prec(precision)
+    M, K = A.shape
+    N = B.shape[1]
+    P = C.shape[1]
+    A, B, C = _c(A, dt), _c(B, dt), _c(C, dt)
+    D = np.empty((M, P), dt)
+    rc = getattr(lib(), f"ft_oracle_b2b_gemm_{precision}")(M, N, K, P, _p(A), _p(B), _p(C), _p(D))
+    if rc:
+        raise RuntimeError(f"oracle b2b_gemm failed: {rc}")
+    return D

@@ -368,3 +368,22 @@ def test_p13b_linear_rnn_layer_one_is_cumsum_of_projection():
     ys = oracle.stacked_rnn(p["x"], p["W"])
     ref = np.cumsum(p["x"].astype(np.float64) @ p["W"][0].astype(np.float64), axis=1)
     np.testing.assert_allclose(ys[:, 0], ref, rtol=1e-13, atol=1e-13)
+
+
+# --------------------------------------------------------------------------- P14 (Table 6 B2B)
+@pytest.mark.parametrize("M,N,K,P", [(7, 13, 5, 3), (128, 256, 64, 64), (3, 1, 2, 4)])
+def test_p14_b2b_gemm_associativity(M, N, K, P):
+    """P14: D = (A@B)@C equals A@(B@C) (associativity — a different evaluation order, through
+    numpy), within fp64 rounding."""
+    g = ftgen.b2b_inputs(M, N, K, P, 31, "f32")
+    D = oracle.b2b_gemm(g["A"], g["B"], g["C"])
+    A, B, C = (g[k].astype(np.float64) for k in ("A", "B", "C"))
+    np.testing.assert_allclose(D, A @ (B @ C), rtol=1e-12, atol=1e-12)
+
+
+def test_p14b_b2b_gemm_identity_reduces_to_gemm():
+    """P14(b): with N = P and C = I, D = A@B (the second product is the identity)."""
+    g = ftgen.b2b_inputs(9, 16, 8, 16, 32, "f32")
+    D = oracle.b2b_gemm(g["A"], g["B"], np.eye(16))
+    np.testing.assert_array_equal(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64)) if False else \
+        np.testing.assert_allclose(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64), rtol=0, atol=1e-14)
