@@ -447,3 +447,25 @@ FT_API long long ft_wavefront_cells(int kind, int depth, int len_a, int len_b, i
     }
     return p.ncells;
 }
+
+FT_API ft_status ft_b2b_gemm_fwd(int M, int N, int K, int P, ft_dtype dt, const void* A,
+                                 const void* B, const void* C, float* D, void* stream) {
+    if (dt != FT_F32 && dt != FT_BF16) return fail(FT_ERR_INVALID_ARGUMENT, "unknown dtype");
+    if (M <= 0 || N <= 0 || K <= 0 || P <= 0)
+        return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    REQUIRE_PTR(A, "A");
+    REQUIRE_PTR(B, "B");
+    REQUIRE_PTR(C, "C");
+    REQUIRE_PTR(D, "D");
+    if (dt != FT_BF16 || K != 64 || P != 64 || M % 128 != 0 || N % 128 != 0)
+        return fail(FT_ERR_UNSUPPORTED,
+                    "b2b GEMM supports bf16 with K = P = 64 (Table 6) and M, N multiples of 128");
+    if ((long long)M * 64 >= (1ll << 31) || (long long)N >= (1ll << 30))
+        return fail(FT_ERR_UNSUPPORTED, "problem too large for 32-bit coordinates");
+    ft_status st = check_device();
+    if (st != FT_OK) return st;
+    std::string err;
+    cudaError_t e = ft::launch_b2b_gemm(M, N, A, B, C, D, static_cast<cudaStream_t>(stream), &err);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, err.empty() ? cudaGetErrorString(e) : err);
+    return FT_OK;
+}

@@ -39,6 +39,9 @@ cudaError_t launch_wavefront_f32(const Problem& p, const Tensors& t, cudaStream_
                                  std::string* err);
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
                                   std::string* err);
+// NEXT-4 back-to-back GEMMs (b2b_gemm.cu): D[M][64] = (A[M][64] @ B[64][N]) @ C[N][64]
+cudaError_t launch_b2b_gemm(int M, int N, const void* A, const void* B, const void* C, float* D,
+                            cudaStream_t s, std::string* err);
 // a5 weight-resident mode (wavefront_resident.cu): slab width 16/32 when the weights fit, else 0
 int resident_bnu(const Problem& p, int nsm);
 cudaError_t launch_wavefront_resident(const Problem& p, const Tensors& t, cudaStream_t s, int bnu,

@@ -29,6 +29,7 @@ EXPORTS = (
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
     "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
     "ft_stacked_rnn_workspace_size", "ft_stacked_rnn_fwd",
+    "ft_b2b_gemm_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells",
@@ -76,6 +77,8 @@ def lib():
         L.ft_stacked_rnn_workspace_size.argtypes = [_c_int] * 5
         L.ft_stacked_rnn_fwd.restype = _c_int
         L.ft_stacked_rnn_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 3 + [_c_vp, _c_size, _c_vp]
+        L.ft_b2b_gemm_fwd.restype = _c_int
+        L.ft_b2b_gemm_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 4 + [_c_vp]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         _lib = L
@@ -140,6 +143,10 @@ def ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace, works
                        stream) -> int:
     return lib().ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace,
                                     workspace_bytes, stream)
+
+
+def ft_b2b_gemm_fwd(M, N, K, P, dt, A, B, C, D, stream) -> int:
+    return lib().ft_b2b_gemm_fwd(M, N, K, P, dt, A, B, C, D, stream)
 
 
 def ft_dilated_rnn_fwd(batch, seq, hidden, depth, dilations, dt, x, W, U, b, y, h_n, c_n, h_all,
@@ -291,3 +298,15 @@ def stacked_rnn(x, W, stream=None, workspace=None):
     check(ft_stacked_rnn_fwd(B, T, H, D, dt, _ptr(x), _ptr(W), _ptr(ys), ws.data_ptr(), ws.numel(),
                              _stream_ptr(stream)))
     return ys
+
+
+def b2b_gemm(A, B, C, stream=None):
+    """Back-to-back GEMMs (Table 6): D = (A @ B) @ C, one fused tcgen05 kernel.
+    A [M][64], B [64][N], C [N][64] bf16 CUDA tensors → D [M][64] fp32."""
+    torch = _torch()
+    M, K = A.shape
+    N = B.shape[1]
+    P = C.shape[1]
+    D = torch.empty((M, P), dtype=torch.float32, device=A.device)
+    check(ft_b2b_gemm_fwd(M, N, K, P, _dt(A), _ptr(A), _ptr(B), _ptr(C), _ptr(D), _stream_ptr(stream)))
+    return D

@@ -333,3 +333,19 @@ def test_bf16_cuda_graph_capture_replay():
     torch.cuda.synchronize()
     ref = oracle.stacked_lstm(p2["x"], p1["W"], p1["U"], p1["b"])
     _check(out, ref, torch.bfloat16, OUT, ctx="graph")
+
+
+# ------------------------------------------------------------------------- NEXT-4: B2B GEMMs
+@pytest.mark.parametrize("M,N", [(128, 128), (256, 512), (1024, 4096), (384, 128)])
+def test_bf16_b2b_gemm(M, N):
+    """Table 6 back-to-back GEMMs (K = P = 64) fused in one tcgen05 kernel vs the fp64 oracle."""
+    g = ftgen.b2b_inputs(M, N, 64, 64, 1919 + M + N, "bf16")
+    A, B, C = (dev(g[k], torch.bfloat16) for k in ("A", "B", "C"))
+    D = ft.b2b_gemm(A, B, C)
+    torch.cuda.synchronize()
+    _check({"D": D}, {"D": oracle.b2b_gemm(g["A"], g["B"], g["C"])}, torch.bfloat16, ("D",), ctx="b2b")
+
+
+def test_b2b_gemm_unsupported_shapes():
+    assert ft.ft_b2b_gemm_fwd(128, 128, 32, 64, ft.FT_BF16, 1 << 20, 1 << 20, 1 << 20, 1 << 20, None) == ft.FT_ERR_UNSUPPORTED
+    assert ft.ft_b2b_gemm_fwd(100, 128, 64, 64, ft.FT_BF16, 1 << 20, 1 << 20, 1 << 20, 1 << 20, None) == ft.FT_ERR_UNSUPPORTED

@@ -385,5 +385,4 @@ def test_p14b_b2b_gemm_identity_reduces_to_gemm():
     """P14(b): with N = P and C = I, D = A@B (the second product is the identity)."""
     g = ftgen.b2b_inputs(9, 16, 8, 16, 32, "f32")
     D = oracle.b2b_gemm(g["A"], g["B"], np.eye(16))
-    np.testing.assert_array_equal(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64)) if False else \
-        np.testing.assert_allclose(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64), rtol=0, atol=1e-14)
+    np.testing.assert_allclose(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64), rtol=0, atol=1e-14)
