@@ -108,8 +108,8 @@ b2b_gemm_kernel(const __grid_constant__ B2Maps M, int N, float* __restrict__ D) 
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            mbar_wait(a_full, 0);
+        {  // the whole warp (warp-uniform waits keep the MMA descriptors in uniform registers)
+            mbar_wait_warp(a_full, 0);
             tc_fence_after();
             const uint64_t ad = make_sdesc(smem_u32(sA), 16, 1024);
             // B chunk: MN-major, two 64-n atoms 8 KiB apart (LBO), 8-k groups 1 KiB (SBO)
@@ -120,32 +120,39 @@ b2b_gemm_kernel(const __grid_constant__ B2Maps M, int N, float* __restrict__ D) 
             const uint64_t sd0 = make_sdesc(smem_u32(sS), 16, 1024);
             auto gemm1 = [&](int j) {
                 const int st = j % NSTAGE;
-                mbar_wait(&bc_full[st], (uint32_t)((j / NSTAGE) & 1));
-                mbar_wait(&s_tfree[j & 1], (uint32_t)(((j >> 1) & 1) ^ 1));
+                mbar_wait_warp(&bc_full[st], (uint32_t)((j / NSTAGE) & 1));
+                mbar_wait_warp(&s_tfree[j & 1], (uint32_t)(((j >> 1) & 1) ^ 1));
                 tc_fence_after();
-                const uint64_t bd = bd0 + (uint64_t)((st * B_B) >> 4);
+                if (elect_one()) {
+                    const uint64_t bd = bd0 + (uint64_t)((st * B_B) >> 4);
 #pragma unroll
-                for (int kk = 0; kk < KD / 16; ++kk)
-                    umma_f16(tmem + (uint32_t)((j & 1) * NC), ad + (uint64_t)((kk * 32) >> 4),
-                             bd + (uint64_t)((kk * 2048) >> 4), IDESC1, kk != 0);
-                umma_commit(&s_full[j & 1]);
+                    for (int kk = 0; kk < KD / 16; ++kk)
+                        umma_f16(tmem + (uint32_t)((j & 1) * NC), ad + (uint64_t)((kk * 32) >> 4),
+                                 bd + (uint64_t)((kk * 2048) >> 4), IDESC1, kk != 0);
+                    umma_commit(&s_full[j & 1]);
+                }
+                __syncwarp();
             };
             gemm1(0);
             for (int j = 0; j < NJ; ++j) {
                 if (j + 1 < NJ) gemm1(j + 1);
-                mbar_wait(&ss_full[j & 1], (uint32_t)((j >> 1) & 1));
+                mbar_wait_warp(&ss_full[j & 1], (uint32_t)((j >> 1) & 1));
                 tc_fence_after();
-                const int st = j % NSTAGE;
-                const uint64_t cd = cd0 + (uint64_t)((st * C_B) >> 4);
-                const uint64_t sd = sd0 + (uint64_t)(((j & 1) * S_B) >> 4);
+                if (elect_one()) {
+                    const int st = j % NSTAGE;
+                    const uint64_t cd = cd0 + (uint64_t)((st * C_B) >> 4);
+                    const uint64_t sd = sd0 + (uint64_t)(((j & 1) * S_B) >> 4);
 #pragma unroll
-                for (int kk = 0; kk < NC / 16; ++kk)
-                    umma_f16(tmem + 256u, sd + (uint64_t)((((kk >> 2) * 16384) + (kk & 3) * 32) >> 4),
-                             cd + (uint64_t)((kk * 2048) >> 4), IDESC2, (j | kk) != 0);
-                umma_commit(&ss_free[j & 1]);
-                umma_commit(&bc_empty[st]);
+                    for (int kk = 0; kk < NC / 16; ++kk)
+                        umma_f16(tmem + 256u, sd + (uint64_t)((((kk >> 2) * 16384) + (kk & 3) * 32) >> 4),
+                                 cd + (uint64_t)((kk * 2048) >> 4), IDESC2, (j | kk) != 0);
+                    umma_commit(&ss_free[j & 1]);
+                    umma_commit(&bc_empty[st]);
+                }
+                __syncwarp();
             }
-            umma_commit(d_full);
+            if (elect_one()) umma_commit(d_full);
+            __syncwarp();
         }
     } else {
         const int q = warp & 3, row = q * 32 + lane;

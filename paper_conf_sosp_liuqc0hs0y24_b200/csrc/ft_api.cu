@@ -333,6 +333,57 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     return FT_OK;
 }
 
+FT_API size_t ft_stacked_lstm_layerwise_workspace_size(int batch, int seq, int hidden, int depth,
+                                                       ft_dtype dt) {
+    if (dt != FT_BF16 || depth <= 0 || depth > FT_MAX_DEPTH || batch <= 0 || seq <= 0 || hidden <= 0 ||
+        hidden % 64 != 0)
+        return 0;
+    return ft::layerwise_ws_bytes(batch, seq, hidden);
+}
+
+FT_API ft_status ft_stacked_lstm_layerwise_fwd(int batch, int seq, int hidden, int depth, ft_dtype dt,
+                                               const void* x, const void* W, const void* U,
+                                               const float* b, void* y, void* h_n, float* c_n,
+                                               void* h_all, float* c_all, void* workspace,
+                                               size_t workspace_bytes, void* stream) {
+    if (dt != FT_F32 && dt != FT_BF16) return fail(FT_ERR_INVALID_ARGUMENT, "unknown dtype");
+    if (batch <= 0 || seq <= 0 || hidden <= 0 || depth <= 0)
+        return fail(FT_ERR_INVALID_ARGUMENT, "every dimension must be > 0");
+    if (depth > FT_MAX_DEPTH) return fail(FT_ERR_UNSUPPORTED, "depth > FT_MAX_DEPTH");
+    if (dt != FT_BF16) return fail(FT_ERR_UNSUPPORTED, "the layer-sequential schedule is bf16 only");
+    if (hidden % 64 != 0) return fail(FT_ERR_UNSUPPORTED, "bf16 path requires hidden % 64 == 0");
+    if ((long long)batch * seq * 4 * hidden >= (1ll << 31) ||
+        (long long)seq * hidden * ((batch + 127) / 128 * 128) / 64 >= (1ll << 31))
+        return fail(FT_ERR_UNSUPPORTED, "problem too large for 32-bit GEMM / TMA coordinates");
+    REQUIRE_PTR(x, "x");
+    REQUIRE_PTR(W, "W");
+    REQUIRE_PTR(U, "U");
+    REQUIRE_PTR(b, "b");
+    REQUIRE_PTR(y, "y");
+    REQUIRE_PTR(h_n, "h_n");
+    REQUIRE_PTR(c_n, "c_n");
+    OPTIONAL_PTR(h_all, "h_all");
+    OPTIONAL_PTR(c_all, "c_all");
+    const size_t need = ft::layerwise_ws_bytes(batch, seq, hidden);
+    if (!workspace) return fail(FT_ERR_INVALID_ARGUMENT, "workspace is NULL");
+    if (!aligned16(workspace)) return fail(FT_ERR_INVALID_ARGUMENT, "workspace not 16-byte aligned");
+    if (workspace_bytes < need)
+        return fail(FT_ERR_WORKSPACE_TOO_SMALL, "workspace_bytes " + std::to_string(workspace_bytes) +
+                                                    " < required " + std::to_string(need));
+    ft_status st = check_device();
+    if (st != FT_OK) return st;
+    int dev = 0, nsm = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    std::string why;
+    if (ft::layerwise_supported(batch, hidden, nsm, &why) != 0) return fail(FT_ERR_UNSUPPORTED, why);
+    std::string err;
+    cudaError_t e = ft::launch_layerwise(batch, seq, hidden, depth, x, W, U, b, y, h_n, c_n, h_all,
+                                         c_all, workspace, static_cast<cudaStream_t>(stream), &err);
+    if (e != cudaSuccess) return fail(FT_ERR_CUDA, err.empty() ? cudaGetErrorString(e) : err);
+    return FT_OK;
+}
+
 FT_API size_t ft_stacked_rnn_workspace_size(int batch, int seq, int hidden, int depth, ft_dtype dt) {
     if (depth <= 0 || depth > FT_MAX_DEPTH) return 0;
     int ones[FT_MAX_DEPTH];

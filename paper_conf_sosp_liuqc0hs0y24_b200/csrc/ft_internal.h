@@ -47,4 +47,12 @@ int resident_bnu(const Problem& p, int nsm);
 cudaError_t launch_wavefront_resident(const Problem& p, const Tensors& t, cudaStream_t s, int bnu,
                                       std::string* err);
 
+// NEXT-2 layer-sequential comparison schedule (layerwise.cu): per layer a hoisted input
+// projection GEMM (cuBLAS) + a U-resident recurrent kernel.
+int layerwise_supported(int B, int H, int nsm, std::string* why);
+size_t layerwise_ws_bytes(int B, int T, int H);
+cudaError_t launch_layerwise(int B, int T, int H, int D, const void* x, const void* W, const void* U,
+                             const float* b, void* y, void* h_n, float* c_n, void* h_all,
+                             float* c_all, void* ws, cudaStream_t s, std::string* err);
+
 }  // namespace ft

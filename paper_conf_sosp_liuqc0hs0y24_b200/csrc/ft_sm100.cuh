@@ -59,6 +59,31 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     }
 }
 
+// Warp-collective bounded wait for the MMA-issuing warp: every lane polls and the warp leaves
+// together, so the wait's outcome is warp-uniform.  This keeps the MMA loop's descriptors in
+// uniform registers: with a single-lane wait the compiler moves them to vector registers and
+// re-loads the SAME uniform registers (R2UR) before every UTCHMMA, a write-after-read hazard that
+// serialises issue with tensor-core dispatch — measured 114 vs 65 cycles per M128 N128 K16 MMA
+// (tools/umma_bench.cu, DESIGN.md §6 "MMA issue").
+__device__ __forceinline__ void mbar_wait_warp(uint64_t* bar, uint32_t parity) {
+    if (__all_sync(0xffffffffu, mbar_try_wait(bar, parity))) return;
+    const uint64_t t0 = globaltimer_ns();
+    for (;;) {
+#pragma unroll 1
+        for (int it = 0; it < 64; ++it)
+            if (__all_sync(0xffffffffu, mbar_try_wait(bar, parity))) return;
+        if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
+    }
+}
+// One elected lane of a converged warp (the lowest active lane: lane 0 when all are active).
+__device__ __forceinline__ bool elect_one() {
+    uint32_t p;
+    asm volatile(
+        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\tselp.u32 %0, 1, 0, e;\n\t}"
+        : "=r"(p));
+    return p != 0;
+}
+
 // ------------------------------------------------------------------------------ proxies
 __device__ __forceinline__ void fence_proxy_async_global() {
     asm volatile("fence.proxy.async.global;" ::: "memory");

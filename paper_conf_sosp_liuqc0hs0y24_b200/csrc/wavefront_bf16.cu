@@ -280,50 +280,56 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
         const int nchunks = segments(P, tl, seg) * kchunks;
         FT_TR_DECL;
         FT_TR_BEGIN();
-        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
         FT_TR_END(TR_M_TEMPTY);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * C::BN);
         for (int c = 0; c < nchunks; ++c) {
             FT_TR_BEGIN();
-            mbar_wait(&full[stage], phase);
+            mbar_wait_warp(&full[stage], phase);
             FT_TR_END(TR_M_FULL);
             tc_fence_after();
-            if (P.debug & 4) {  // timing experiment: no MMA, hand the slot straight back
-                if constexpr (CG == 1) {
-                    mbar_arrive(&empty[stage]);
+            if (elect_one()) {
+                if (P.debug & 4) {  // timing experiment: no MMA, hand the slot straight back
+                    if constexpr (CG == 1) {
+                        mbar_arrive(&empty[stage]);
+                    } else {
+                        mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 0));
+                        mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 1));
+                    }
                 } else {
-                    mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 0));
-                    mbar_arrive_cluster(mapa_shared(smem_u32(&empty[stage]), 1));
-                }
-            } else {
-            const uint64_t ad = adesc0 + (uint64_t)((stage * C::A_BYTES) >> 4);
-            const uint64_t bd = bdesc0 + (uint64_t)((stage * C::B_BYTES) >> 4);
+                    const uint64_t ad = adesc0 + (uint64_t)((stage * C::A_BYTES) >> 4);
+                    const uint64_t bd = bdesc0 + (uint64_t)((stage * C::B_BYTES) >> 4);
 #pragma unroll
-            for (int kk = 0; kk < BK / UK; ++kk)
-                umma_f16_cg<CG>(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
-                                bd + (uint64_t)((kk * UK * C::WROW) >> 4), C::IDESC, (c | kk) != 0);
-            umma_commit_cg<CG>(&empty[stage]);
+                    for (int kk = 0; kk < BK / UK; ++kk)
+                        umma_f16_cg<CG>(d_tmem, ad + (uint64_t)((kk * UK * 2) >> 4),
+                                        bd + (uint64_t)((kk * UK * C::WROW) >> 4), C::IDESC, (c | kk) != 0);
+                    umma_commit_cg<CG>(&empty[stage]);
+                }
             }
+            __syncwarp();
             if (++stage == C::STAGES) {
                 stage = 0;
                 phase ^= 1;
             }
         }
-        if (P.debug & 4) {
-            if constexpr (CG == 1) {
-                mbar_arrive(&tfull[acc]);
+        if (elect_one()) {
+            if (P.debug & 4) {
+                if constexpr (CG == 1) {
+                    mbar_arrive(&tfull[acc]);
+                } else {
+                    mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 0));
+                    mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 1));
+                }
             } else {
-                mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 0));
-                mbar_arrive_cluster(mapa_shared(smem_u32(&tfull[acc]), 1));
+                umma_commit_cg<CG>(&tfull[acc]);
             }
-        } else {
-            umma_commit_cg<CG>(&tfull[acc]);
         }
+        __syncwarp();
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
-    FT_TR_FLUSH(true);
+    FT_TR_FLUSH((threadIdx.x & 31) == 0);
 }
 
 // ------------------------------------------------------------------------------ epilogue
@@ -688,7 +694,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     if (warp == 0) {
         if (lane == 0) run_producer<CG, U, true>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
-        if (lane == 0 && rank == 0) run_mma<CG, U>(P, tmem_base, sA, sB, full, empty, tfull, tempty);
+        if (rank == 0) run_mma<CG, U>(P, tmem_base, sA, sB, full, empty, tfull, tempty);  // whole warp
     } else if (warp == 10) {
         if (lane == 0) run_producer<CG, U, false>(P, T, M, sA, sB, full, empty, rank);
     } else {

@@ -134,8 +134,8 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
             }
         }
     } else if (warp == 1) {
-        if (lane == 0) {
-            mbar_wait(wbar, 0);
+        {  // the whole warp (warp-uniform waits keep the MMA descriptors in uniform registers)
+            mbar_wait_warp(wbar, 0);
             tc_fence_after();
             const uint64_t adesc0 = make_sdesc(smem_u32(sA), 16, 1024);
             // weights: MN-major, BNU-wide swizzle atoms; gate atoms GATE_BYTES apart (LBO),
@@ -144,26 +144,30 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
             int stage = 0, acc = 0;
             uint32_t phase = 0, acc_phase = 0;
             for (int t = 0; t < P.L0; ++t) {
-                mbar_wait(&tempty[acc], acc_phase ^ 1);
+                mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
                 tc_fence_after();
                 const uint32_t d_tmem = tmem_base + (uint32_t)(acc * C::N);
                 const int nch = (t > 0 ? 2 : 1) * KCH;
                 for (int c = 0; c < nch; ++c) {
-                    mbar_wait(&full[stage], phase);
+                    mbar_wait_warp(&full[stage], phase);
                     tc_fence_after();
-                    const uint64_t ad = adesc0 + (uint64_t)((stage * C::A_BYTES) >> 4);
-                    const uint64_t bd = bdesc0 + (uint64_t)((c * C::WCHUNK) >> 4);
+                    if (elect_one()) {
+                        const uint64_t ad = adesc0 + (uint64_t)((stage * C::A_BYTES) >> 4);
+                        const uint64_t bd = bdesc0 + (uint64_t)((c * C::WCHUNK) >> 4);
 #pragma unroll
-                    for (int kk = 0; kk < RBK / 16; ++kk)
-                        umma_f16(d_tmem, ad + (uint64_t)((kk * 32) >> 4),
-                                 bd + (uint64_t)((kk * 16 * C::SW) >> 4), C::IDESC, (c | kk) != 0);
-                    umma_commit(&empty[stage]);
+                        for (int kk = 0; kk < RBK / 16; ++kk)
+                            umma_f16(d_tmem, ad + (uint64_t)((kk * 32) >> 4),
+                                     bd + (uint64_t)((kk * 16 * C::SW) >> 4), C::IDESC, (c | kk) != 0);
+                        umma_commit(&empty[stage]);
+                    }
+                    __syncwarp();
                     if (++stage == C::STAGES) {
                         stage = 0;
                         phase ^= 1;
                     }
                 }
-                umma_commit(&tfull[acc]);
+                if (elect_one()) umma_commit(&tfull[acc]);
+                __syncwarp();
                 acc ^= 1;
                 if (acc == 0) acc_phase ^= 1;
             }

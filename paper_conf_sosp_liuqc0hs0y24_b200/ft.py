@@ -29,6 +29,7 @@ EXPORTS = (
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
     "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
     "ft_stacked_rnn_workspace_size", "ft_stacked_rnn_fwd",
+    "ft_stacked_lstm_layerwise_workspace_size", "ft_stacked_lstm_layerwise_fwd",
     "ft_b2b_gemm_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
@@ -77,6 +78,10 @@ def lib():
         L.ft_stacked_rnn_workspace_size.argtypes = [_c_int] * 5
         L.ft_stacked_rnn_fwd.restype = _c_int
         L.ft_stacked_rnn_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 3 + [_c_vp, _c_size, _c_vp]
+        L.ft_stacked_lstm_layerwise_workspace_size.restype = _c_size
+        L.ft_stacked_lstm_layerwise_workspace_size.argtypes = [_c_int] * 5
+        L.ft_stacked_lstm_layerwise_fwd.restype = _c_int
+        L.ft_stacked_lstm_layerwise_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 9 + [_c_vp, _c_size, _c_vp]
         L.ft_b2b_gemm_fwd.restype = _c_int
         L.ft_b2b_gemm_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 4 + [_c_vp]
         L.ft_wavefront_cells.restype = _c_ll
@@ -143,6 +148,16 @@ def ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace, works
                        stream) -> int:
     return lib().ft_stacked_rnn_fwd(batch, seq, hidden, depth, dt, x, W, ys, workspace,
                                     workspace_bytes, stream)
+
+
+def ft_stacked_lstm_layerwise_workspace_size(batch, seq, hidden, depth, dt):
+    return lib().ft_stacked_lstm_layerwise_workspace_size(batch, seq, hidden, depth, dt)
+
+
+def ft_stacked_lstm_layerwise_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n, c_n, h_all,
+                                  c_all, workspace, workspace_bytes, stream) -> int:
+    return lib().ft_stacked_lstm_layerwise_fwd(batch, seq, hidden, depth, dt, x, W, U, b, y, h_n,
+                                               c_n, h_all, c_all, workspace, workspace_bytes, stream)
 
 
 def ft_b2b_gemm_fwd(M, N, K, P, dt, A, B, C, D, stream) -> int:
@@ -249,6 +264,30 @@ def stacked_lstm(x, W, U, b, want_all=False, dilations=None, stream=None, worksp
                                 _ptr(y), _ptr(h_n), _ptr(c_n), _ptr(h_all), _ptr(c_all),
                                 ws.data_ptr(), ws.numel(), sp)
     check(st)
+    r = dict(y=y, h_n=h_n, c_n=c_n)
+    if want_all:
+        r.update(h_all=h_all, c_all=c_all)
+    return r
+
+
+def stacked_lstm_layerwise(x, W, U, b, want_all=False, stream=None, workspace=None):
+    """The layer-sequential comparison schedule (NEXT-2): same inputs and outputs as
+    `stacked_lstm` (bf16 only), computed one layer after another with a hoisted input GEMM."""
+    torch = _torch()
+    B, T, H = x.shape
+    D = W.shape[0]
+    dt = _dt(x)
+    dev = x.device
+    y = torch.empty((B, T, H), dtype=x.dtype, device=dev)
+    h_n = torch.empty((B, D, H), dtype=x.dtype, device=dev)
+    c_n = torch.empty((B, D, H), dtype=torch.float32, device=dev)
+    h_all = torch.empty((B, D, T, H), dtype=x.dtype, device=dev) if want_all else None
+    c_all = torch.empty((B, D, T, H), dtype=torch.float32, device=dev) if want_all else None
+    nbytes = ft_stacked_lstm_layerwise_workspace_size(B, T, H, D, dt)
+    ws = (workspace or Workspace()).get(nbytes, dev)
+    check(ft_stacked_lstm_layerwise_fwd(B, T, H, D, dt, _ptr(x), _ptr(W), _ptr(U), _ptr(b), _ptr(y),
+                                        _ptr(h_n), _ptr(c_n), _ptr(h_all), _ptr(c_all),
+                                        ws.data_ptr(), ws.numel(), _stream_ptr(stream)))
     r = dict(y=y, h_n=h_n, c_n=c_n)
     if want_all:
         r.update(h_all=h_all, c_all=c_all)

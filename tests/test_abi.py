@@ -87,6 +87,27 @@ def test_dilation_and_grid_validation():
     assert ft.ft_grid_rnn_fwd(**g) == ft.FT_ERR_INVALID_ARGUMENT
 
 
+@pytest.mark.parametrize("over,code", [
+    (dict(batch=0), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(dt=7), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(dt=ft.FT_F32), ft.FT_ERR_UNSUPPORTED),
+    (dict(hidden=96), ft.FT_ERR_UNSUPPORTED),
+    (dict(depth=65), ft.FT_ERR_UNSUPPORTED),
+    (dict(U=None), ft.FT_ERR_INVALID_ARGUMENT),
+    (dict(workspace_bytes=16), ft.FT_ERR_WORKSPACE_TOO_SMALL),
+])
+def test_layerwise_validation(over, code):
+    """NEXT-2 entry point: same argument checks as ft_stacked_lstm_fwd, bf16 only."""
+    a = dict(batch=4, seq=8, hidden=64, depth=2, dt=ft.FT_BF16, x=FAKE, W=FAKE, U=FAKE, b=FAKE,
+             y=FAKE, h_n=FAKE, c_n=FAKE, h_all=None, c_all=None, workspace=FAKE,
+             workspace_bytes=1 << 40, stream=None)
+    a.update(over)
+    assert ft.ft_stacked_lstm_layerwise_fwd(**a) == code
+    n = ft.ft_stacked_lstm_layerwise_workspace_size(256, 100, 1024, 16, ft.FT_BF16)
+    assert n >= 256 * 100 * 4 * 1024 * 4 + 2 * 256 * 100 * 1024 * 2  # fp32 Z + two layer outputs
+    assert ft.ft_stacked_lstm_layerwise_workspace_size(256, 100, 1024, 16, ft.FT_F32) == 0
+
+
 def test_valid_call_without_gpu_reports_cuda_error():
     import torch
     if torch.cuda.is_available():

@@ -349,3 +349,44 @@ def test_bf16_b2b_gemm(M, N):
 def test_b2b_gemm_unsupported_shapes():
     assert ft.ft_b2b_gemm_fwd(128, 128, 32, 64, ft.FT_BF16, 1 << 20, 1 << 20, 1 << 20, 1 << 20, None) == ft.FT_ERR_UNSUPPORTED
     assert ft.ft_b2b_gemm_fwd(100, 128, 64, 64, ft.FT_BF16, 1 << 20, 1 << 20, 1 << 20, 1 << 20, None) == ft.FT_ERR_UNSUPPORTED
+
+
+# ------------------------------------------------------------------------- NEXT-2 layer-sequential
+def _run_layerwise(p, want_all=False):
+    x, W, U = dev(p["x"], torch.bfloat16), dev(p["W"], torch.bfloat16), dev(p["U"], torch.bfloat16)
+    b = dev(p["b"], torch.float32)
+    r = ft.stacked_lstm_layerwise(x, W, U, b, want_all=want_all)
+    torch.cuda.synchronize()
+    return r
+
+
+@pytest.mark.parametrize("B,T,H,D", [(1, 1, 64, 1), (5, 4, 64, 3), (130, 6, 128, 2), (64, 9, 256, 4),
+                                     (256, 3, 320, 2)])
+def test_bf16_layerwise_matches_oracle(B, T, H, D):
+    """NEXT-2: the layer-sequential schedule (hoisted cuBLAS input GEMM + U-resident recurrent
+    kernel) computes the same nest (legal order: Table 4's distances are non-negative)."""
+    p = ftgen.stacked_inputs(B, T, H, D, 808 + B + H, "bf16")
+    got = _run_layerwise(p, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"layerwise {B,T,H,D}")
+
+
+@pytest.mark.slow
+def test_bf16_layerwise_C3_sampled_rows():
+    c = ftgen.CONFIGS["C3"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C3"), "bf16")
+    got = _run_layerwise(p)
+    rows = ftgen.sample_rows(c["batch"], 0, 1)[:4]
+    _check(got, _oracle_stacked(p, rows=rows), torch.bfloat16, OUT, rows=rows, ctx="layerwise C3")
+
+
+def test_layerwise_unsupported_shapes():
+    z = torch.zeros(16, device="cuda")
+    # batch 1024 at hidden 1024 needs 8 x 64 = 512 co-resident CTAs
+    n = ft.ft_stacked_lstm_layerwise_workspace_size(1024, 2, 1024, 1, ft.FT_BF16)
+    ws = torch.empty(n, dtype=torch.uint8, device="cuda")
+    st = ft.ft_stacked_lstm_layerwise_fwd(1024, 2, 1024, 1, ft.FT_BF16, *[z.data_ptr()] * 7, None, None,
+                                          ws.data_ptr(), n, None)
+    assert st == ft.FT_ERR_UNSUPPORTED, ft.ft_last_error()
+    st = ft.ft_stacked_lstm_layerwise_fwd(4, 2, 64, 1, ft.FT_F32, *[z.data_ptr()] * 7, None, None,
+                                          ws.data_ptr(), n, None)
+    assert st == ft.FT_ERR_UNSUPPORTED
