@@ -9,7 +9,9 @@ hidden 1024, bf16 operands / fp32 accumulation — the configuration the metric 
 A step = one full forward of the nest (every cell of every diagonal) over one batch — one
 ft_stacked_lstm_fwd call (flag reset + the persistent wavefront kernel).  Multi-GPU: the batch
 `map` is sharded (each rank runs 256 sequences: weak scaling), no collective in the data path;
---gather adds an NCCL gather of y to rank 0 (the north star's optional output gather).
+--gather [nccl|fused] adds the north star's final output gather of y to rank 0: `nccl` calls
+torch.distributed.gather after each forward; `fused` maps rank 0's output buffers into every rank
+(CUDA IPC / NVLink P2P) so the kernel epilogue writes there directly.
 
 Prints ONE JSON line on rank 0.  Timing: W untimed warm-ups, then K steps bracketed by
 barrier + cuda synchronize, CUDA events on the launching stream, max over ranks.  L2: the
@@ -261,11 +263,15 @@ def run_ours(args):
     outs = {"y": torch.empty((B, T, H), dtype=bf, device=dev),
             "h_n": torch.empty((B, D, H), dtype=bf, device=dev),
             "c_n": torch.empty((B, D, H), dtype=torch.float32, device=dev)}
-    from paper_conf_sosp_liuqc0hs0y24_b200.shard import gather_rows
+    from paper_conf_sosp_liuqc0hs0y24_b200.shard import PeerGather, gather_rows
+    if args.gather == "fused" and world > 1:
+        # NEXT-1: y / h_n / c_n stored by the kernel epilogue straight into rank 0's buffers
+        peer = PeerGather(B * world, T, H, D, bf, dev, dst=0)
+        outs = peer.local()
 
     def step():
         ft.stacked_lstm(x, W, U, b, workspace=ws, out=outs)
-        if args.gather and world > 1:  # the final output gather of y to rank 0 (NCCL / NVLink)
+        if args.gather == "nccl" and world > 1:  # the final output gather of y to rank 0 (NCCL)
             gather_rows(outs["y"], B * world, dst=0)
 
     stream = torch.cuda.current_stream()
@@ -372,7 +378,7 @@ def run_ours(args):
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
         "data": "synthetic (ftgen splitmix64: x~U(-1,1), W,U,b~U(+-1/sqrt(H)), bf16 RNE)",
-        "config": workload_config(n_gpus),
+        "config": dict(workload_config(n_gpus), gather=args.gather),
         "tensor_pipe_pct_of_peak": 100.0 * roofline["frac"],
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
         "gpu_launches": 2 * args.steps, "clocks": clocks,
@@ -391,7 +397,9 @@ def main():
     ap.add_argument("--steps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    ap.add_argument("--gather", action="store_true", help="NCCL-gather y to rank 0 each step")
+    ap.add_argument("--gather", nargs="?", const="nccl", default="none", choices=["none", "nccl", "fused"],
+                    help="gather y to rank 0 each step: nccl = torch.distributed.gather after the kernel; "
+                         "fused = the kernel stores into rank 0's buffer over NVLink (NEXT-1)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:

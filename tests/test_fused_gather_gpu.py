@@ -1,0 +1,58 @@
+"""NEXT-1: the output gather fused into the kernel (shard.PeerGather).
+
+Two ranks (processes) share cuda:0 — gpurun gives one GPU; on an NVSwitch node the same code maps
+a peer GPU's memory over NVLink.  Rank 0 allocates the full y / h_n / c_n; each rank passes its row
+slice of rank 0's buffers straight to ft_stacked_lstm_fwd, so the epilogue stores land in rank 0's
+memory.  The gathered result must equal a single-process run of the whole batch (rows are
+independent — Table 1; both runs use the same 128-row tile shape, so bitwise)."""
+import os
+import socket
+
+import pytest
+import torch
+
+pytestmark = pytest.mark.gpu
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, out_path):
+    import numpy as np
+    import torch.distributed as dist
+    import ftgen
+    from paper_conf_sosp_liuqc0hs0y24_b200 import ft
+    from paper_conf_sosp_liuqc0hs0y24_b200.shard import PeerGather, shard_rows
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    Bt, T, H, D = 128, 5, 128, 3
+    p = ftgen.stacked_inputs(Bt, T, H, D, 4242, "bf16")
+    bf = torch.bfloat16
+    W, U = (torch.from_numpy(p[k]).cuda().to(bf) for k in ("W", "U"))
+    b = torch.from_numpy(p["b"]).cuda()
+    a, e = shard_rows(Bt, world, rank)
+    x = torch.from_numpy(np.ascontiguousarray(p["x"][a:e])).cuda().to(bf)
+    peer = PeerGather(Bt, T, H, D, bf, "cuda:0", dst=0)
+    ft.stacked_lstm(x, W, U, b, out=peer.local())
+    full = peer.done()
+    if rank == 0:
+        xf = torch.from_numpy(p["x"]).cuda().to(bf)
+        ref = ft.stacked_lstm(xf, W, U, b)
+        torch.cuda.synchronize()
+        ok = {k: bool(torch.equal(full[k], ref[k])) for k in ("y", "h_n", "c_n")}
+        with open(out_path, "w") as f:
+            f.write(repr(ok))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_fused_gather_two_ranks_one_gpu(tmp_path, cuda_device):
+    import torch.multiprocessing as mp
+    out = str(tmp_path / "ok.txt")
+    mp.spawn(_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    res = eval(open(out).read())
+    assert res == {"y": True, "h_n": True, "c_n": True}, res
