@@ -23,4 +23,15 @@ run_seq(130, 4, 128, 2, torch.bfloat16)               # streaming, CTA pair
 run_seq(20, 7, 128, 3, torch.bfloat16, dil=[1, 2, 3])
 run_grid(3, 3, 4, 64, 2, torch.bfloat16)
 run_grid(3, 3, 4, 16, 2, torch.float32)
+os.environ["FT_TILE_UNITS"] = "32"
+run_seq(130, 4, 128, 2, torch.bfloat16, resident="0")  # CTA pair, 32-unit tiles
+os.environ.pop("FT_TILE_UNITS")
+p = ftgen.stacked_inputs(130, 4, 128, 2, 1, "bf16")       # NEXT-2 layer-sequential schedule
+a = [torch.from_numpy(p[k]).to(dev, torch.bfloat16) for k in ("x", "W", "U")] + [torch.from_numpy(p["b"]).to(dev)]
+ft.stacked_lstm_layerwise(*a, want_all=True)
+xs = torch.from_numpy(p["x"]).to(dev, torch.bfloat16)     # NEXT-3 linear RNN
+ft.stacked_rnn(xs, a[1][:, 0].contiguous())
+g = ftgen.b2b_inputs(256, 256, 64, 64, 1, "bf16")          # NEXT-4 back-to-back GEMMs
+ft.b2b_gemm(*[torch.from_numpy(g[k]).to(dev, torch.bfloat16) for k in ("A", "B", "C")])
+torch.cuda.synchronize()
 print("sanitize cases done")
