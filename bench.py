@@ -141,6 +141,17 @@ def host_cores():
         return os.cpu_count() or 1
 
 
+def load_ncu_tensor_pct():
+    """ncu's tensor-pipe active % of the committed C3 capture (profiles/latest_C3_ncu_summary.json)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "latest_C3_ncu_summary.json")) as f:
+            d = json.load(f)
+        m = d.get("metrics", d)
+        return m["sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed"]["value"]
+    except (OSError, KeyError, ValueError, TypeError):
+        return None
+
+
 def pin_oracle_threads():
     # torchrun exports OMP_NUM_THREADS=1; the CPU baseline uses every host core it may run on.
     # Must run before oracle/liboracle.so is first loaded (OpenMP reads it at initialisation).
@@ -159,15 +170,35 @@ def oracle_rate(p, rows, tsteps=None):
     return dt, rows * frac
 
 
+def host_info():
+    """The CPU the oracle baseline ran on: model, logical CPUs, affinity."""
+    model = None
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    try:
+        aff = len(os.sched_getaffinity(0))
+    except AttributeError:
+        aff = None
+    return {"cpu_model": model, "logical_cpus": os.cpu_count(), "affinity_cpus": aff}
+
+
 def cpu_baseline(p):
     pin_oracle_threads()
     import oracle
     n = oracle.num_threads()
     dt, seqs = oracle_rate(p, n)
-    return {"value": seqs / dt, "unit": UNIT, "cores": n, "kind": "oracle",
-            "sample": f"{n} of 256 batch rows of C3 (full depth 16, seq 100; rows are independent "
-                      f"by the batch map, P6), f32 instantiation of oracle/ft_oracle.c, OpenMP over "
-                      f"rows, {dt:.1f} s wall"}
+    flop_per_seq = 16.0 * p["W"].shape[-1] ** 2 * p["x"].shape[1] * p["W"].shape[0]
+    return dict({"value": seqs / dt, "unit": UNIT, "cores": n, "kind": "oracle",
+                 "gflops": seqs * flop_per_seq / dt / 1e9,
+                 "sample": f"{n} of 256 batch rows of C3 (full depth 16, seq 100; rows are independent "
+                           f"by the batch map, P6), f32 instantiation of oracle/ft_oracle.c, OpenMP over "
+                           f"rows, {dt:.1f} s wall"}, **host_info())
 
 
 # ----------------------------------------------------------------------------- inputs
@@ -214,8 +245,8 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": total / args.steps * 1e3,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
         "data": "synthetic", "config": workload_config(1),
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": nthr, "kind": "oracle",
-                         "sample": sample},
+        "cpu_baseline": dict({"value": value, "unit": UNIT, "cores": nthr, "kind": "oracle",
+                              "sample": sample}, **host_info()),
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -317,7 +348,19 @@ def run_ours(args):
                 "flops_per_launch": flops,
                 "launch_ms_mean": mean_call_s * 1e3,
                 "note": "launch duration = one ft_stacked_lstm_fwd call: counter reset + x pack "
-                        "(52 MB) + the persistent wavefront kernel, CUDA events on the launch stream"}
+                        "(52 MB) + the persistent wavefront kernel, CUDA events on the launch stream",
+                "launch_ms_median": statistics.median(call_ms), "launch_ms_min": min(call_ms)}
+    # bound time of the binding roofline row (SURVEY d.2: tensor 4.26 ms, HBM 4.10 ms at C3) and
+    # the DRAM side from the committed ncu capture
+    t_tensor = flops / (peak_b * 1e12)
+    roofline["t_bound_ms"] = t_tensor * 1e3
+    tr = roofline["traffic"]
+    if tr and hbm:
+        roofline["hbm"] = {"bytes_per_launch_ncu": tr, "peak_GBps": hbm,
+                           "frac": tr / mean_call_s / 1e9 / hbm}
+    ncu_pct = load_ncu_tensor_pct()
+    if ncu_pct is not None:
+        roofline["ncu_tensor_pipe_active_pct"] = ncu_pct
 
     # the same achieved rate against the tensor peak at the clock the run actually had (148 SMs x
     # 8192 dense bf16 FLOP/clk/SM x the median SM clock sampled during the timed region): the
