@@ -41,7 +41,7 @@ def lib():
     if _lib is None:
         build()
         _lib = ctypes.CDLL(LIB_PATH)
-        for sfx in ("f64", "f32"):
+        for sfx in ("f64", "f32", "bf16emu"):
             for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell", "stacked_rnn",
                          "b2b_gemm"):
                 fn = getattr(_lib, f"ft_oracle_{name}_{sfx}")
@@ -60,7 +60,7 @@ def _p(a):
 def _prec(precision):
     if precision == "f64":
         return np.float64
-    if precision == "f32":
+    if precision in ("f32", "bf16emu"):  # bf16emu: diagnostic, float with h rounded to bf16 per cell
         return np.float32
     raise ValueError(precision)
 

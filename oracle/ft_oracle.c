@@ -28,7 +28,10 @@
  * + hp[k]·U[k][n] for k ascending.  The k-outer / n-inner loop below performs exactly that
  * sequence of additions for every output (it only changes which output is updated next).
  *
- * Precision: REAL = double (the parity reference) or float (CPU timing instantiation).
+ * Precision: REAL = double (the parity reference) or float (CPU timing instantiation), plus a
+ * DIAGNOSTIC-ONLY third build, _bf16emu: float with h rounded to bf16 (round-to-nearest-even)
+ * after every cell, mirroring the rounding point of the bf16 GPU path (R20; SURVEY
+ * §8(c) c.4).  It separates kernel bugs from precision effects and is never the judged reference.
  * Parallelism: OpenMP over the batch map only (fully parallel, Table 1 map, L126); this does
  * not change any output's arithmetic.
  */
@@ -42,13 +45,24 @@
 
 #define ORACLE_EXPORT __attribute__((visibility("default")))
 
+/* float -> nearest bf16 (ties to even), returned as float; finite inputs only */
+static float oracle_round_bf16(float v) {
+    unsigned int u;
+    memcpy(&u, &v, sizeof(u));
+    u += 0x7FFFu + ((u >> 16) & 1u);
+    u &= 0xFFFF0000u;
+    memcpy(&v, &u, sizeof(v));
+    return v;
+}
+
 /* ---------------------------------------------------------------------------------------- */
-/* instantiate everything twice: _f64 (parity) and _f32 (timing)                            */
+/* instantiate three times: _f64 (parity), _f32 (timing), _bf16emu (diagnostic)             */
 /* ---------------------------------------------------------------------------------------- */
 #define REAL double
 #define SFX(name) name##_f64
 #define EXPF exp
 #define TANHF tanh
+#define ROUND_H(v) (v)
 #include "ft_oracle_impl.h"
 #undef REAL
 #undef SFX
@@ -60,10 +74,18 @@
 #define EXPF expf
 #define TANHF tanhf
 #include "ft_oracle_impl.h"
+#undef SFX
+#undef ROUND_H
+
+/* diagnostic: float with h rounded to bf16 after every LSTM cell */
+#define SFX(name) name##_bf16emu
+#define ROUND_H(v) oracle_round_bf16(v)
+#include "ft_oracle_impl.h"
 #undef REAL
 #undef SFX
 #undef EXPF
 #undef TANHF
+#undef ROUND_H
 
 ORACLE_EXPORT int ft_oracle_num_threads(void) {
 #ifdef _OPENMP

@@ -390,3 +390,18 @@ def test_layerwise_unsupported_shapes():
     st = ft.ft_stacked_lstm_layerwise_fwd(4, 2, 64, 1, ft.FT_F32, *[z.data_ptr()] * 7, None, None,
                                           ws.data_ptr(), n, None)
     assert st == ft.FT_ERR_UNSUPPORTED
+
+
+def test_bf16_vs_bf16_emulating_oracle_diagnostic():
+    """c.4 diagnostic: the GPU bf16 path against the oracle's bf16-emulating build (h rounded to bf16
+    at the same point as the kernel).  What remains is summation order and the MUFU activations; it
+    must be within the judged tolerance too.  The judged reference stays the fp64 oracle."""
+    c = ftgen.CONFIGS["C2"]
+    p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C2"), "bf16")
+    got = _run_stacked(p, torch.bfloat16)
+    emu = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="bf16emu")
+    ref = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"])
+    for k in OUT:
+        g = host(got[k])
+        e_emu, e_ref = normrel(g, emu[k].astype(np.float64)), normrel(g, ref[k])
+        assert e_emu <= BF16_TOL and e_ref <= BF16_TOL, (k, e_emu, e_ref)

@@ -386,3 +386,28 @@ def test_p14b_b2b_gemm_identity_reduces_to_gemm():
     g = ftgen.b2b_inputs(9, 16, 8, 16, 32, "f32")
     D = oracle.b2b_gemm(g["A"], g["B"], np.eye(16))
     np.testing.assert_allclose(D, g["A"].astype(np.float64) @ g["B"].astype(np.float64), rtol=0, atol=1e-14)
+
+
+# --------------------------------------------------------------------------- c.4 diagnostic mode
+def test_bf16emu_rounds_h_like_the_generator_once():
+    """The diagnostic _bf16emu build rounds each cell's h to bf16 (RNE).  On one cell (T = D = 1)
+    that is exactly round_bf16 of the f32 build's h — checked against ftgen.round_bf16, an
+    independent implementation of the same rounding (numpy, in the input generator)."""
+    p = ftgen.stacked_inputs(3, 1, 48, 1, 91, "bf16", scale=2.0)
+    f32 = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="f32", want_all=True)
+    emu = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="bf16emu", want_all=True)
+    assert np.array_equal(emu["h_all"], ftgen.round_bf16(f32["h_all"]).astype(np.float32))
+    assert np.array_equal(emu["c_all"], f32["c_all"])  # c is never rounded (R20)
+
+
+def test_bf16emu_within_precision_headroom():
+    """P11 in the diagnostic mode: bf16 emulation vs the fp64 reference stays well inside the 2e-2
+    normwise tolerance at the judged distribution, and every stored h is a bf16 value."""
+    p = ftgen.stacked_inputs(2, 12, 256, 4, 92, "bf16")
+    ref = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], want_all=True)
+    emu = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision="bf16emu", want_all=True)
+    for k in ("y", "h_n", "c_n"):
+        err = np.max(np.abs(emu[k] - ref[k])) / np.max(np.abs(ref[k]))
+        assert 0 < err < 5e-3, (k, err)
+    bits = emu["h_all"].view(np.uint32)
+    assert np.all((bits & 0xFFFF) == 0)
