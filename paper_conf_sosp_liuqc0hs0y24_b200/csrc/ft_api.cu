@@ -216,6 +216,7 @@ ft_status seq_fwd(int batch, int seq, int hidden, int depth, const int* dil, ft_
 }  // namespace
 
 namespace ft {
+void set_last_error(const std::string& msg) { g_last_error = msg; }
 long long c_ring_elems(const Problem& p) {
     if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * p.B * p.H;
     return (long long)p.D * 2 * p.L1 * p.B * p.H + (long long)p.D * p.L0 * 2 * p.B * p.H;
@@ -230,6 +231,7 @@ FT_API const char* ft_status_string(ft_status s) {
         case FT_ERR_INVALID_ARGUMENT: return "FT_ERR_INVALID_ARGUMENT";
         case FT_ERR_UNSUPPORTED: return "FT_ERR_UNSUPPORTED";
         case FT_ERR_CUDA: return "FT_ERR_CUDA";
+        case FT_ERR_NCCL: return "FT_ERR_NCCL";
         case FT_ERR_WORKSPACE_TOO_SMALL: return "FT_ERR_WORKSPACE_TOO_SMALL";
     }
     return "FT_ERR_UNKNOWN";

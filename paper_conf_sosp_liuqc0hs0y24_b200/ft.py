@@ -18,7 +18,7 @@ import os
 PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(PKG, "libft.so")
 
-FT_OK, FT_ERR_INVALID_ARGUMENT, FT_ERR_UNSUPPORTED, FT_ERR_CUDA = 0, 1, 2, 3
+FT_OK, FT_ERR_INVALID_ARGUMENT, FT_ERR_UNSUPPORTED, FT_ERR_CUDA, FT_ERR_NCCL = 0, 1, 2, 3, 4
 FT_ERR_WORKSPACE_TOO_SMALL = 5
 FT_F32, FT_BF16 = 0, 1
 FT_MAX_DEPTH = 64
@@ -34,6 +34,7 @@ EXPORTS = (
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells",
+    "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
 )
 
 
@@ -84,6 +85,12 @@ def lib():
         L.ft_stacked_lstm_layerwise_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 9 + [_c_vp, _c_size, _c_vp]
         L.ft_b2b_gemm_fwd.restype = _c_int
         L.ft_b2b_gemm_fwd.argtypes = [_c_int] * 5 + [_c_vp] * 4 + [_c_vp]
+        L.ft_comm_create.restype = _c_int
+        L.ft_comm_create.argtypes = [_c_int, _c_vp, ctypes.POINTER(_c_vp)]
+        L.ft_comm_gather.restype = _c_int
+        L.ft_comm_gather.argtypes = [_c_vp, _c_vp, _c_vp, _c_vp, _c_int, _c_vp]
+        L.ft_comm_destroy.restype = _c_int
+        L.ft_comm_destroy.argtypes = [_c_vp]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         _lib = L
@@ -187,6 +194,27 @@ def ft_wavefront_cells(kind, depth, len_a, len_b=1):
     buf = (ctypes.c_int * (4 * n))()
     lib().ft_wavefront_cells(kind, depth, len_a, len_b, ctypes.cast(buf, _c_vp), n)
     return [tuple(buf[4 * k:4 * k + 4]) for k in range(n)]
+
+
+def ft_comm_create(devices):
+    """Returns (status, comm handle) for an NCCL communicator over `devices` (one process)."""
+    arr = _int_array(devices)
+    out = _c_vp()
+    st = lib().ft_comm_create(len(devices), ctypes.cast(arr, _c_vp), ctypes.byref(out))
+    return st, out.value
+
+
+def ft_comm_gather(comm, send_ptrs, recv_ptr, nbytes, root, stream_ptrs):
+    n = len(send_ptrs)
+    send = (_c_vp * n)(*send_ptrs)
+    sizes = (_c_size * n)(*nbytes)
+    streams = (_c_vp * n)(*stream_ptrs)
+    return lib().ft_comm_gather(comm, ctypes.cast(send, _c_vp), recv_ptr, ctypes.cast(sizes, _c_vp),
+                                root, ctypes.cast(streams, _c_vp))
+
+
+def ft_comm_destroy(comm):
+    return lib().ft_comm_destroy(comm)
 
 
 def check(status: int):

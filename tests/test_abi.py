@@ -108,6 +108,21 @@ def test_layerwise_validation(over, code):
     assert ft.ft_stacked_lstm_layerwise_workspace_size(256, 100, 1024, 16, ft.FT_F32) == 0
 
 
+def test_comm_validation():
+    """Multi-GPU gather ABI: argument checks before any NCCL / CUDA work."""
+    L = ft.lib()
+    assert L.ft_comm_create(1, None, None) == ft.FT_ERR_INVALID_ARGUMENT  # out is NULL
+    st, comm = ft.ft_comm_create([])
+    assert st == ft.FT_ERR_INVALID_ARGUMENT and comm is None
+    assert ft.ft_comm_gather(None, [FAKE], FAKE, [16], 0, [None]) == ft.FT_ERR_INVALID_ARGUMENT
+    assert ft.ft_comm_destroy(None) == ft.FT_OK
+    assert ft.status_string(ft.FT_ERR_NCCL) == "FT_ERR_NCCL"
+    import torch
+    if not torch.cuda.is_available():
+        st, comm = ft.ft_comm_create([0])
+        assert st == ft.FT_ERR_CUDA and comm is None
+
+
 def test_valid_call_without_gpu_reports_cuda_error():
     import torch
     if torch.cuda.is_available():

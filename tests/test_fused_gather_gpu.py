@@ -56,3 +56,21 @@ def test_fused_gather_two_ranks_one_gpu(tmp_path, cuda_device):
     mp.spawn(_worker, args=(2, _free_port(), out), nprocs=2, join=True)
     res = eval(open(out).read())
     assert res == {"y": True, "h_n": True, "c_n": True}, res
+
+
+def test_comm_gather_abi_one_device(cuda_device):
+    """ft_comm_create / ft_comm_gather / ft_comm_destroy on the one GPU gpurun gives: the root's
+    own slice is copied into place (the NCCL send/recv leg needs >= 2 devices).  On an 8-GPU node
+    the same call gathers every device's y slice to the root over NVLink."""
+    from paper_conf_sosp_liuqc0hs0y24_b200 import ft
+    st, comm = ft.ft_comm_create([0])
+    assert st == ft.FT_OK, ft.ft_last_error()
+    src = torch.arange(4096, dtype=torch.float32, device="cuda")
+    dst = torch.zeros_like(src)
+    s = torch.cuda.current_stream().cuda_stream
+    st = ft.ft_comm_gather(comm, [src.data_ptr()], dst.data_ptr(), [src.numel() * 4], 0, [s])
+    assert st == ft.FT_OK, ft.ft_last_error()
+    torch.cuda.synchronize()
+    assert torch.equal(src, dst)
+    assert ft.ft_comm_gather(comm, [src.data_ptr()], dst.data_ptr(), [16], 1, [s]) == ft.FT_ERR_INVALID_ARGUMENT
+    assert ft.ft_comm_destroy(comm) == ft.FT_OK
