@@ -210,25 +210,32 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
         FT_TR_DECL;
         if constexpr (!kWeights) {
-            // the producer cells of this tile (Table 4 dependence vectors): one acquire each of
-            // their (cell, m-block) counters before any activation load of the tile
             FT_TR_ADD(TR_TILES, 1);
-            long long prod[3];
-            producers(P, tl.cell, prod);
-            FT_TR_BEGIN();
             if (rank == 0) FT_EV(tile, 0);
-            if (!(P.debug & 1)) {
+            if (P.debug & 256) {  // A/B experiment: acquire every producer before any load
+                long long prod[3];
+                producers(P, tl.cell, prod);
 #pragma unroll
                 for (int q = 0; q < 3; ++q)
                     if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
+                fence_proxy_async_global();
             }
-            FT_TR_END(TR_P_FLAG);
-            if (rank == 0) FT_EV(tile, 1);
-            fence_proxy_async_global();
         }
         int si = 0, kc = 0;
         for (int c = 0; c < nchunks; ++c) {
             const Segment sg = pick(seg, si);
+            if constexpr (!kWeights) {
+                // the segment's producer cell (Table 4 dependence vectors): one acquire of its
+                // (cell, m-block) counter before the segment's first activation load, so inputs
+                // that are ready (x, the layer below) stream in while a later producer finishes
+                if (kc == 0 && sg.scell >= 0 && !(P.debug & 1)) {
+                    FT_TR_BEGIN();
+                    wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
+                    FT_TR_END(TR_P_FLAG);
+                    fence_proxy_async_global();
+                }
+                if (c == 0 && rank == 0) FT_EV(tile, 1);
+            }
             if constexpr (kWeights) FT_TR_BEGIN();
             mbar_wait(&empty[stage], phase ^ 1);
             if constexpr (kWeights) FT_TR_END(TR_P_EMPTY);

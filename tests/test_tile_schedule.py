@@ -1,0 +1,121 @@
+"""Tile-to-worker assignment of the persistent streaming kernel, simulated on the host.
+
+The kernel enumerates tiles in the wavefront order of the product scheduler (ft_wavefront_cells,
+the same __host__ __device__ code), `tiles_per_cell` consecutive tiles per cell, and worker w (a
+CTA or CTA pair) processes tiles w, w + nw, w + 2nw, ... in order.  A simulation of in-order
+workers that may start a tile only when its producer cells (Table 4 dependence vectors; the
+dilation stride, L331) are complete must finish — the deadlock-freedom argument of DESIGN.md §6 —
+and, in an event model with a dependency latency, must keep the critical path.  No GPU needed.
+"""
+import pytest
+
+from paper_conf_sosp_liuqc0hs0y24_b200 import build, ft
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    build.build()
+
+
+def _producers(kind, cell, dil):
+    _, d, i, j = cell
+    if kind == 0:
+        out = [(d - 1, i, 0)] if d > 0 else []
+        if i >= dil[d]:
+            out.append((d, i - dil[d], 0))
+        return out
+    out = [(d - 1, i, j)] if d > 0 else []
+    if i > 0:
+        out.append((d, i - 1, j))
+    if j > 0:
+        out.append((d, i, j - 1))
+    return out
+
+
+def _owner(ntiles, nw):
+    """The kernel's static assignment: tile g of the wavefront sequence -> worker g mod nw."""
+    return [g % nw for g in range(ntiles)]
+
+
+def _simulate(kind, D, La, Lb, dil, tpc, nw):
+    """Unit-time rounds: each worker completes its next tile when the tile's producer cells are
+    complete.  Returns the number of rounds (raises on deadlock)."""
+    cells = ft.ft_wavefront_cells(kind, D, La, Lb)
+    ordinal = {(c[1], c[2], c[3]): o for o, c in enumerate(cells)}
+    owner = _owner(len(cells) * tpc, nw)
+    queues = [[] for _ in range(nw)]
+    for g, w in enumerate(owner):
+        assert 0 <= w < nw
+        queues[w].append(g)                      # appended in g order = the worker's order
+    left = [tpc] * len(cells)
+    heads = [0] * nw
+    rounds = 0
+    remaining = len(owner)
+    while remaining:
+        done_now = []
+        for w in range(nw):
+            if heads[w] < len(queues[w]):
+                g = queues[w][heads[w]]
+                cell = cells[g // tpc]
+                if all(left[ordinal[p]] == 0 for p in _producers(kind, cell, dil or [1] * D)):
+                    done_now.append((w, g))
+        assert done_now, "deadlock: no worker can make progress"
+        for w, g in done_now:
+            heads[w] += 1
+            left[g // tpc] -= 1
+        remaining -= len(done_now)
+        rounds += 1
+    return rounds
+
+
+@pytest.mark.parametrize("kind,D,La,Lb,dil,tpc,nw", [
+    (0, 6, 30, 1, [1, 2, 4, 8, 16, 32], 16, 74),   # C4-like, 32-unit tiles, 74 CTA pairs
+    (0, 16, 12, 1, None, 16, 74),                   # C3-like depth, short sequence
+    (0, 4, 12, 1, [1, 1, 3, 2], 8, 10),
+    (0, 5, 7, 1, None, 4, 3),                       # fewer workers than tiles per cell
+    (1, 3, 4, 5, None, 16, 148),                    # grid, 1-CTA workers
+    (1, 4, 6, 3, None, 2, 5),
+])
+def test_assignment_is_deadlock_free(kind, D, La, Lb, dil, tpc, nw):
+    _simulate(kind, D, La, Lb, dil, tpc, nw)
+
+
+def _event_makespan(kind, D, La, Lb, dil, tpc, nw, tau=1.0, lat=2.0):
+    """Event model of the persistent kernel: a worker runs its tiles in order, each takes `tau`
+    (the MMA), and may start only `lat` (counter propagation + operand loads) after its producer
+    cells completed.  Returns the makespan."""
+    cells = ft.ft_wavefront_cells(kind, D, La, Lb)
+    ordinal = {(c[1], c[2], c[3]): o for o, c in enumerate(cells)}
+    owner = _owner(len(cells) * tpc, nw)
+    queues = [[] for _ in range(nw)]
+    for g, w in enumerate(owner):
+        queues[w].append(g)
+    left, end, free, heads = [tpc] * len(cells), [0.0] * len(cells), [0.0] * nw, [0] * nw
+    for _ in range(len(owner)):
+        best = None
+        for w in range(nw):
+            if heads[w] < len(queues[w]):
+                g = queues[w][heads[w]]
+                ps = [ordinal[p] for p in _producers(kind, cells[g // tpc], dil or [1] * D)]
+                if all(left[p] == 0 for p in ps):
+                    st = max([free[w]] + [end[p] + lat for p in ps])
+                    if best is None or st < best[0]:
+                        best = (st, w, g)
+        assert best is not None, "deadlock"
+        st, w, g = best
+        free[w] = st + tau
+        heads[w] += 1
+        left[g // tpc] -= 1
+        end[g // tpc] = max(end[g // tpc], st + tau)
+    return max(free)
+
+
+def test_assignment_keeps_the_critical_path():
+    """C4's shape (6 layers, dilations 1..32, 16 tiles per cell, 74 CTA pairs) at T = 30: with
+    per-tile time tau and dependency latency lat, round-robin finishes in the critical path
+    (T + D - 1 steps of tau + lat) — no critical tile waits behind work that has slack.  (A
+    variant reserving workers for the dilation-1 layer measured slower on the GPU: DESIGN §6.)"""
+    dil = [1, 2, 4, 8, 16, 32]
+    T, D, tau, lat = 30, 6, 1.0, 2.0
+    span = _event_makespan(0, D, T, 1, dil, 16, 74, tau, lat)
+    assert span <= (T + D - 1) * (tau + lat), span
