@@ -60,10 +60,12 @@ enum TraceSlot {
 };
 __device__ unsigned long long g_trace[1024 * TR_SLOTS];
 // per-tile event timestamps (%globaltimer, ns) of the leader CTA: 0 wait start, 1 deps ready,
-// 2 A loads issued, 3 MMA done (epilogue saw tfull), 4 counter released
+// 2 A loads issued, 3 MMA done (epilogue saw tfull), 4 counter released, 5 last producer flag
+// acquired, 6 MMA warp got the accumulator, 7 MMA warp issued the last chunk
 constexpr int EV_MAX_TILES = 65536;
-__device__ unsigned long long g_events[EV_MAX_TILES * 5];
-#define FT_EV(tile, k) do { if ((tile) < EV_MAX_TILES) g_events[(tile) * 5 + (k)] = globaltimer_ns(); } while (0)
+constexpr int EV_K = 8;
+__device__ unsigned long long g_events[EV_MAX_TILES * EV_K];
+#define FT_EV(tile, k) do { if ((tile) < EV_MAX_TILES) g_events[(tile) * EV_K + (k)] = globaltimer_ns(); } while (0)
 // register accumulators, flushed once per role (keeps the instrumented loops lean)
 #define FT_TR_ROLE unsigned long long _acc[TR_SLOTS] = {0}
 #define FT_TR_DECL long long _tr0 = 0
@@ -232,6 +234,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                     FT_TR_BEGIN();
                     wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
                     FT_TR_END(TR_P_FLAG);
+                    if (rank == 0) FT_EV(tile, 5);
                     fence_proxy_async_global();
                 }
                 if (c == 0 && rank == 0) FT_EV(tile, 1);
@@ -289,6 +292,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
         FT_TR_BEGIN();
         mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
         FT_TR_END(TR_M_TEMPTY);
+        if ((threadIdx.x & 31) == 0) FT_EV(tile, 6);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * C::BN);
         for (int c = 0; c < nchunks; ++c) {
@@ -320,6 +324,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
                 phase ^= 1;
             }
         }
+        if ((threadIdx.x & 31) == 0) FT_EV(tile, 7);
         if (elect_one()) {
             if (P.debug & 4) {
                 if constexpr (CG == 1) {
@@ -900,7 +905,7 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_trace(unsigned lo
 extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned long long* host, int ntiles) {
     if (ntiles > EV_MAX_TILES) ntiles = EV_MAX_TILES;
     cudaDeviceSynchronize();
-    if (cudaMemcpyFromSymbol(host, g_events, (size_t)ntiles * 5 * sizeof(unsigned long long)) != cudaSuccess) return -1;
+    if (cudaMemcpyFromSymbol(host, g_events, (size_t)ntiles * EV_K * sizeof(unsigned long long)) != cudaSuccess) return -1;
     return ntiles;
 }
 #endif

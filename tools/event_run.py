@@ -17,9 +17,10 @@ for _ in range(4): ft.stacked_lstm(*a, workspace=ws, dilations=dil)
 torch.cuda.synchronize()
 D, T, NT = c["depth"], c["seq"], c["hidden"] // nt_units
 ntiles = D * T * NT
-buf = (ctypes.c_ulonglong * (ntiles * 5))()
+EV_K = 8
+buf = (ctypes.c_ulonglong * (ntiles * EV_K))()
 L.ft_debug_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
 L.ft_debug_events(buf, ntiles)
-ev = np.array(buf[:], dtype=np.float64).reshape(ntiles, 5)
+ev = np.array(buf[:], dtype=np.float64).reshape(ntiles, EV_K)
 np.save(f"gpurun_out/events_{name.lower()}.npy", ev)
 print("saved", ev.shape)
