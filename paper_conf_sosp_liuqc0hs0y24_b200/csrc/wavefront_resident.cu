@@ -108,11 +108,18 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
             int stage = 0;
             uint32_t phase = 0;
             for (int t = 0; t < P.L0; ++t) {
-                if (d > 0) wait_flag_geq(T.flags + cell_lin(P, d - 1, t, 0), target);
-                if (t > 0) wait_flag_geq(T.flags + cell_lin(P, d, t - 1, 0), target);
-                fence_proxy_async_global();
                 const int nch = (t > 0 ? 2 : 1) * KCH;
                 for (int c = 0; c < nch; ++c) {
+                    // acquire each half's producer just before its first chunk: the input half
+                    // (layer below / x) streams in while the recurrent producer still runs
+                    if (c == 0 && d > 0) {
+                        wait_flag_geq(T.flags + cell_lin(P, d - 1, t, 0), target);
+                        fence_proxy_async_global();
+                    }
+                    if (c == KCH) {
+                        wait_flag_geq(T.flags + cell_lin(P, d, t - 1, 0), target);
+                        fence_proxy_async_global();
+                    }
                     mbar_wait(&empty[stage], phase ^ 1);
                     mbar_arrive_expect_tx(&full[stage], C::A_BYTES);
                     const uint32_t dst = smem_u32(sA + stage * C::A_BYTES);
