@@ -405,3 +405,15 @@ def test_bf16_vs_bf16_emulating_oracle_diagnostic():
         g = host(got[k])
         e_emu, e_ref = normrel(g, emu[k].astype(np.float64)), normrel(g, ref[k])
         assert e_emu <= BF16_TOL and e_ref <= BF16_TOL, (k, e_emu, e_ref)
+
+
+@pytest.mark.parametrize("B,Lx,Ly,H,D", [(5, 4, 3, 64, 2), (128, 5, 5, 128, 3), (100, 2, 7, 64, 2),
+                                         (33, 1, 4, 64, 2), (64, 6, 1, 192, 2)])
+def test_bf16_grid_shapes(B, Lx, Ly, H, D):
+    """Grid (batch <= 128, 1-CTA tiles): odd diagonal groups, one-axis grids, ragged batches."""
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, 1717 + B + Lx, "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx=f"grid {B,Lx,Ly,H,D}")
