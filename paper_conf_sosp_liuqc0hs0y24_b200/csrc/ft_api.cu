@@ -218,8 +218,8 @@ ft_status seq_fwd(int batch, int seq, int hidden, int depth, const int* dil, ft_
 namespace ft {
 void set_last_error(const std::string& msg) { g_last_error = msg; }
 long long c_ring_elems(const Problem& p) {
-    if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * p.B * p.H;
-    return (long long)p.D * 2 * p.L1 * p.B * p.H + (long long)p.D * p.L0 * 2 * p.B * p.H;
+    if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * c_slot_elems(p);
+    return ((long long)p.D * 2 * p.L1 + (long long)p.D * p.L0 * 2) * c_slot_elems(p);
 }
 }  // namespace ft
 

@@ -250,17 +250,23 @@ FT_HD int src_rows(const Problem& p, int src) {
 // [ring_off[d], ring_off[d+1]); slot of step t is t mod ring_len_d.  The slot written by
 // (d, t) last held c(d, t - 2s_d), read by (d, t - s_d) — a direct producer of (d, t), so the
 // reuse is ordered by the flag protocol.  KIND_GRID: c^x ring of 2 slots over i
-// ([D][2][Ly][B][H]) and c^y ring of 2 slots over j ([D][Lx][2][B][H]), same argument.
+// ([D][2][Ly] slots) and c^y ring of 2 slots over j ([D][Lx][2] slots), same argument.
+// Inside a slot the layout is [H/4][B][4]: 4 units of one batch row are one 16-byte vector and
+// consecutive batch rows are adjacent, so an epilogue warp (one thread per batch row) loads and
+// stores whole 512-byte runs.  (A [B][H] slot made every warp store 32 partial sectors 4 KiB
+// apart; those stores cost 23 % of C3's energy at the power cap — profiles/r2_power.)
+FT_HD long long c_slot_elems(const Problem& p) { return (long long)((p.H + 3) >> 2) * 4 * p.B; }
+FT_HD long long c_slot_index(const Problem& p, long long slot, int b, int n) {
+    return ((slot * ((p.H + 3) >> 2) + (n >> 2)) * p.B + b) * 4 + (n & 3);
+}
 FT_HD long long c_ring_index(const Problem& p, int d, int i, int j, int a, int b, int n) {
     if (p.kind == KIND_SEQ) {
         const int len = p.ring_off[d + 1] - p.ring_off[d];
-        const long long slot = p.ring_off[d] + i % len;
-        return (slot * p.B + b) * (long long)p.H + n;
+        return c_slot_index(p, p.ring_off[d] + i % len, b, n);
     }
-    if (a == 0)
-        return ((((long long)d * 2 + (i & 1)) * p.L1 + j) * p.B + b) * (long long)p.H + n;
-    const long long base = (long long)p.D * 2 * p.L1 * p.B * p.H;
-    return base + ((((long long)d * p.L0 + i) * 2 + (j & 1)) * p.B + b) * (long long)p.H + n;
+    if (a == 0) return c_slot_index(p, ((long long)d * 2 + (i & 1)) * p.L1 + j, b, n);
+    const long long base = (long long)p.D * 2 * p.L1;
+    return c_slot_index(p, base + ((long long)d * p.L0 + i) * 2 + (j & 1), b, n);
 }
 
 // The cell whose c the tile's epilogue reads (its c-producer), or -1 (zero initial state).

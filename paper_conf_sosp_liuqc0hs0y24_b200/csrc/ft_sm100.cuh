@@ -90,6 +90,12 @@ __device__ __forceinline__ void st_v4_hint(void* p, uint4 v, uint64_t pol) {
                  "r"(v.z), "r"(v.w), "l"(pol)
                  : "memory");
 }
+// 256-bit store (sm_100: STG.256): one whole 32-byte L2 sector per thread
+__device__ __forceinline__ void st_v8_hint(void* p, uint4 a, uint4 b, uint64_t pol) {
+    asm volatile("st.global.L2::cache_hint.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8}, %9;" ::"l"(p),
+                 "r"(a.x), "r"(a.y), "r"(a.z), "r"(a.w), "r"(b.x), "r"(b.y), "r"(b.z), "r"(b.w), "l"(pol)
+                 : "memory");
+}
 __device__ __forceinline__ float4 ld_cg_v4_hint(const void* p, uint64_t pol) {
     float4 v;
     asm volatile("ld.global.cg.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"

@@ -406,10 +406,9 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
             const int n = n0 + u0;
             if (!valid || n >= P.H) continue;
             if (cprod >= 0) {
-                const float4* src = reinterpret_cast<const float4*>(T.c_ring + c_ring_index(P, c.d, ci, cj, 0, b, n));
 #pragma unroll
                 for (int v = 0; v < 4; ++v) {
-                    const float4 t4 = __ldcg(src + v);
+                    const float4 t4 = __ldcg(reinterpret_cast<const float4*>(T.c_ring + c_ring_index(P, c.d, ci, cj, 0, b, n + 4 * v)));
                     z[4 * v] += t4.x;
                     z[4 * v + 1] += t4.y;
                     z[4 * v + 2] += t4.z;
@@ -421,9 +420,10 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
             for (int w = 0; w < 2; ++w)
                 hp[w] = make_uint4(pack_bf16x2(z[8 * w + 0], z[8 * w + 1]), pack_bf16x2(z[8 * w + 2], z[8 * w + 3]),
                                    pack_bf16x2(z[8 * w + 4], z[8 * w + 5]), pack_bf16x2(z[8 * w + 6], z[8 * w + 7]));
-            float4* cdst = reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, 0, b, n));
 #pragma unroll
-            for (int v = 0; v < 4; ++v) __stcg(cdst + v, make_float4(z[4 * v], z[4 * v + 1], z[4 * v + 2], z[4 * v + 3]));
+            for (int v = 0; v < 4; ++v)
+                __stcg(reinterpret_cast<float4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, 0, b, n + 4 * v)),
+                       make_float4(z[4 * v], z[4 * v + 1], z[4 * v + 2], z[4 * v + 3]));
             uint4* hdst = reinterpret_cast<uint4*>((__nv_bfloat16*)T.hb + hb_row(P, row_h, n / 64, b) * 64 + (n % 64));
             __stcg(hdst, hp[0]);
             __stcg(hdst + 1, hp[1]);
@@ -497,11 +497,11 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
         float cp[EPI_UNITS];
         if (cprod >= 0 && valid) {
-            const float4* src = reinterpret_cast<const float4*>(
-                T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n0));
+            const float* src = T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n0);
+            const long long vstride = 4ll * P.B;  // next 4 units of the same batch row
 #pragma unroll
             for (int v = 0; v < EPI_UNITS / 4; ++v) {
-                const float4 t4 = ld_cg_v4_hint(src + v, pol_state);
+                const float4 t4 = ld_cg_v4_hint(reinterpret_cast<const float4*>(src + v * vstride), pol_state);
                 cp[4 * v + 0] = t4.x;
                 cp[4 * v + 1] = t4.y;
                 cp[4 * v + 2] = t4.z;
@@ -566,6 +566,13 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 bg[v] = t3.x; bg[v + 1] = t3.y; bg[v + 2] = t3.z; bg[v + 3] = t3.w;
             }
             float hv[16];
+            if (P.debug & 1024) {  // timing experiment: no gate math (wrong results)
+#pragma unroll
+                for (int v = 0; v < 16; ++v) {
+                    cv[u0 + v] = zf[v] + cp[u0 + v];
+                    hv[v] = zi[v] + zo[v] + zg[v];
+                }
+            } else
 #pragma unroll
             for (int v = 0; v < 16; ++v) {
                 const float ig = sigmoid_approx(zi[v] + bi[v]);
@@ -584,16 +591,15 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                                             pack_bf16x2(hv[8 * w + 6], hv[8 * w + 7]));
             // what downstream cells read — h (blocked SSA buffer hb) and c (ring) — stored per
             // chunk so the stores overlap the next chunk's math
-            if (valid && !(P.debug & 2)) {
+            if (valid && !(P.debug & 512)) {  // bits 512 / 2048 / 4096: timing experiments (no h/c, c, h stores)
                 const int nn = n0 + u0;
                 uint4* hdst = reinterpret_cast<uint4*>(
                     (__nv_bfloat16*)T.hb + hb_row(P, row_h, nn / 64, b) * 64 + (nn % 64));
-                st_v4_hint(hdst + 0, hp[u0 / 8], pol_state);
-                st_v4_hint(hdst + 1, hp[u0 / 8 + 1], pol_state);
-                uint4* cdst = reinterpret_cast<uint4*>(T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn));
+                if (!(P.debug & 4096)) st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
+                float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn);
 #pragma unroll
                 for (int v = 0; v < 4; ++v)
-                    st_v4_hint(cdst + v,
+                    if (!(P.debug & 2048)) st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
                                make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
                                           __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
                                pol_state);

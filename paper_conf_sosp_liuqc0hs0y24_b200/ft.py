@@ -16,7 +16,7 @@ import ctypes
 import os
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "libft.so")
+LIB_PATH = os.environ.get("FT_LIB_PATH") or os.path.join(PKG, "libft.so")  # override: A/B timing of two builds
 
 FT_OK, FT_ERR_INVALID_ARGUMENT, FT_ERR_UNSUPPORTED, FT_ERR_CUDA, FT_ERR_NCCL = 0, 1, 2, 3, 4
 FT_ERR_WORKSPACE_TOO_SMALL = 5
