@@ -79,7 +79,7 @@ def load_traffic():
 class ClockSampler:
     FIELDS = ("timestamp,clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-              "clocks_event_reasons.sw_power_cap,utilization.gpu,power.draw")
+              "clocks_event_reasons.sw_power_cap,utilization.gpu,power.draw.instant,power.limit")
 
     def __init__(self, index):
         self.index = index
@@ -109,12 +109,12 @@ class ClockSampler:
         with open(self.path) as f:
             for line in f:
                 parts = [x.strip() for x in line.split(",")]
-                if len(parts) < 9:
+                if len(parts) < 10:
                     continue
                 try:
                     rows.append(dict(sm=float(parts[1]), smax=float(parts[2]),
                                      hw=parts[3], hwt=parts[4], swt=parts[5], pc=parts[6],
-                                     util=float(parts[7]), pw=float(parts[8])))
+                                     util=float(parts[7]), pw=float(parts[8]), plim=float(parts[9])))
                 except ValueError:
                     continue
         os.unlink(self.path)
@@ -129,7 +129,10 @@ class ClockSampler:
                     reasons.add(name)
         return {"sm_mhz": statistics.median(r["sm"] for r in loaded),
                 "sm_max_mhz": max(r["smax"] for r in loaded), "reasons": sorted(reasons),
+                # instantaneous board power (power.draw is a 1 s average and under-reads a
+                # sub-second timed region); power.limit is the cap sw_power_cap enforces
                 "power_w_median": statistics.median(r["pw"] for r in loaded),
+                "power_limit_w": max(r["plim"] for r in loaded),
                 "samples": len(loaded)}
 
 

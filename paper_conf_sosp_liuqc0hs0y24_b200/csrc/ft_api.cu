@@ -71,6 +71,8 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         p->resident_layers = wbytes <= 64.0 * 1024 * 1024 ? D : 0;
         const char* env = getenv("FT_L2_RESIDENT_LAYERS");  // tuning override
         if (env) p->resident_layers = atoi(env);
+        const char* pe = getenv("FT_L2_PERSIST_LAYERS");  // experiment: persisting L2 window
+        p->persist_layers = pe ? atoi(pe) : 0;
         const char* dbg = getenv("FT_DEBUG");  // timing experiments only
         p->debug = dbg ? atoi(dbg) : 0;
     }

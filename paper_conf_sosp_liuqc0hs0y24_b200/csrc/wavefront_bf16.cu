@@ -247,7 +247,10 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             if constexpr (kWeights) {
                 if (!skipB) {
                     const CUtensorMap* bm = sg.wsel == W_IN ? &M.W : &M.U;
-                    const uint64_t wpol = weight_layer(P, sg.slice) < P.resident_layers ? pol_keep : pol_stream;
+                    const int wl = weight_layer(P, sg.slice);
+                    const uint64_t wpol = (sg.wsel == W_IN && wl < P.persist_layers)
+                                              ? pol_act
+                                              : (wl < P.resident_layers ? pol_keep : pol_stream);
                     tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
                                               fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
                 }
@@ -889,6 +892,28 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     cfg.gridDim = dim3((unsigned)grid);
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    cudaLaunchAttribute attr2[2];
+    if (p.persist_layers > 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM) {
+        // experiment: W[0 .. persist_layers) in a persisting L2 window
+        int maxp = 0, maxw = 0;
+        cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+        cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev);
+        size_t bytes = (size_t)p.persist_layers * 4 * p.H * p.H * 2;
+        if (bytes > (size_t)maxw) bytes = (size_t)maxw;
+        size_t lim = bytes < (size_t)maxp ? bytes : (size_t)maxp;
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
+        if (getenv("FT_L2_PERSIST_VERBOSE"))
+            fprintf(stderr, "persist: max persisting %d B, max window %d B, window %zu B, limit %zu B\n", maxp, maxw, bytes, lim);
+        attr2[0] = attr[0];
+        attr2[1].id = cudaLaunchAttributeAccessPolicyWindow;
+        attr2[1].val.accessPolicyWindow.base_ptr = const_cast<void*>(t.W);
+        attr2[1].val.accessPolicyWindow.num_bytes = bytes;
+        attr2[1].val.accessPolicyWindow.hitRatio = (float)lim / (float)bytes;
+        attr2[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        attr2[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        cfg.attrs = attr2;
+        cfg.numAttrs = 2;
+    }
     e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, p, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
