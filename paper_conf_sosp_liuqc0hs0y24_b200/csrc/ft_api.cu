@@ -71,8 +71,8 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         p->resident_layers = wbytes <= 64.0 * 1024 * 1024 ? D : 0;
         const char* env = getenv("FT_L2_RESIDENT_LAYERS");  // tuning override
         if (env) p->resident_layers = atoi(env);
-        const char* pe = getenv("FT_L2_PERSIST_LAYERS");  // experiment: persisting L2 window
-        p->persist_layers = pe ? atoi(pe) : 0;
+        const char* pe = getenv("FT_L2_PERSIST_LAYERS");  // experiments: force the window's layer count
+        p->persist_layers = pe ? atoi(pe) : -1;            // -1: sized by ft_set_l2_persist (auto)
         const char* dbg = getenv("FT_DEBUG");  // timing experiments only
         p->debug = dbg ? atoi(dbg) : 0;
     }
@@ -218,6 +218,8 @@ ft_status seq_fwd(int batch, int seq, int hidden, int depth, const int* dil, ft_
 }  // namespace
 
 namespace ft {
+static int g_l2_persist_mib = -1;  // ft_set_l2_persist: -1 auto, 0 off, else MiB
+int l2_persist_mib() { return g_l2_persist_mib; }
 void set_last_error(const std::string& msg) { g_last_error = msg; }
 long long c_ring_elems(const Problem& p) {
     if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * c_slot_elems(p);
@@ -226,6 +228,12 @@ long long c_ring_elems(const Problem& p) {
 }  // namespace ft
 
 FT_API int ft_version(void) { return FT_VERSION; }
+
+FT_API ft_status ft_set_l2_persist(int mib) {
+    if (mib < -1) return fail(FT_ERR_INVALID_ARGUMENT, "ft_set_l2_persist: mib must be >= -1");
+    ft::g_l2_persist_mib = mib;
+    return FT_OK;
+}
 
 FT_API const char* ft_status_string(ft_status s) {
     switch (s) {

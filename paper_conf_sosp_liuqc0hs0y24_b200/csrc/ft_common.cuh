@@ -38,8 +38,8 @@ struct Problem {
     int MB, NT;          // m-blocks = ceil(B/BM), n-tiles per axis = ceil(H/BNU)
     int flag_mult;       // counter increments per tile (CTAs per tile: 2 for a tcgen05 CTA pair)
     int resident_layers; // bf16: layers whose weights are kept in L2 (evict_last); others stream
-    int persist_layers;  // bf16 (experiment, env FT_L2_PERSIST_LAYERS): W of the first layers in a
-                         // persisting L2 access-policy window, loaded with EVICT_NORMAL
+    int persist_layers;  // bf16 streaming: W of the first persist_layers layers lie in a persisting
+                         // L2 access-policy window (loaded with EVICT_NORMAL); host side: -1 = auto
     int debug;           // timing experiments only (env FT_DEBUG; results invalid when != 0):
                          // bit 0 skip dependency waits, bit 1 skip the epilogue math/stores;
                          // bit 6 (64) = stress mode: random delays before each counter release

@@ -35,6 +35,7 @@ constexpr int BF16_BM = 128, BF16_BNU = 64;  // tcgen05 path (BK2–BK4)
 // Number of fp32 ring elements the cell state needs.
 long long c_ring_elems(const Problem& p);
 
+int l2_persist_mib();  // ft_set_l2_persist setting (-1 auto, 0 off, else MiB)
 cudaError_t launch_wavefront_f32(const Problem& p, const Tensors& t, cudaStream_t s,
                                  std::string* err);
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,

@@ -799,6 +799,31 @@ bool encode_wt(EncodeTiledFn enc, CUtensorMap* m, const void* base, int H, int k
     return true;
 }
 
+// The device's persisting-L2 set-aside (cudaLimitPersistingL2CacheSize) is raised once to what
+// the window needs and then left alone (it is device-wide; lowering it would evict other users'
+// persisting lines).  Never changed while `s` is being captured into a graph.
+bool persisting_limit_at_least(int dev, size_t bytes, cudaStream_t s) {
+    static size_t set_to[64] = {0};
+    if (dev < 0 || dev >= 64) return false;
+    if (set_to[dev] >= bytes) return true;
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(s, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) {
+        cudaGetLastError();
+        return false;
+    }
+    size_t cur = 0;
+    if (cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize) == cudaSuccess && cur >= bytes) {
+        set_to[dev] = cur;
+        return true;
+    }
+    if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    set_to[dev] = bytes;
+    return true;
+}
+
 template <int CG, int U>
 cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
     using C = KCfg<CG, U>;
@@ -892,29 +917,43 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     cfg.gridDim = dim3((unsigned)grid);
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    // Persisting L2 window over W of the first layers (streaming regime only: the weight set does
+    // not fit in L2, so every diagonal re-reads it from DRAM).  The window's layers are read from
+    // L2 on every diagonal after the first; their TMA loads carry EVICT_NORMAL so the hint does
+    // not fight the window.  C3: DRAM 31.5 -> 28.5 GB per forward, -3 % time at the power cap
+    // (profiles/r2_ab_l2_persist.jsonl).  ft_set_l2_persist() sizes or disables it.
+    Problem q = p;
+    q.persist_layers = 0;
     cudaLaunchAttribute attr2[2];
-    if (p.persist_layers > 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM) {
-        // experiment: W[0 .. persist_layers) in a persisting L2 window
+    if (p.resident_layers == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.persist_layers != 0) {
         int maxp = 0, maxw = 0;
         cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
         cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev);
-        size_t bytes = (size_t)p.persist_layers * 4 * p.H * p.H * 2;
-        if (bytes > (size_t)maxw) bytes = (size_t)maxw;
-        size_t lim = bytes < (size_t)maxp ? bytes : (size_t)maxp;
-        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, lim);
-        if (getenv("FT_L2_PERSIST_VERBOSE"))
-            fprintf(stderr, "persist: max persisting %d B, max window %d B, window %zu B, limit %zu B\n", maxp, maxw, bytes, lim);
-        attr2[0] = attr[0];
-        attr2[1].id = cudaLaunchAttributeAccessPolicyWindow;
-        attr2[1].val.accessPolicyWindow.base_ptr = const_cast<void*>(t.W);
-        attr2[1].val.accessPolicyWindow.num_bytes = bytes;
-        attr2[1].val.accessPolicyWindow.hitRatio = (float)lim / (float)bytes;
-        attr2[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-        attr2[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-        cfg.attrs = attr2;
-        cfg.numAttrs = 2;
+        const size_t layer_bytes = (size_t)4 * p.H * p.H * 2;
+        const long long mib = l2_persist_mib();
+        size_t budget = mib >= 0 ? (size_t)mib << 20 : (size_t)48 << 20;  // auto: 48 MiB (measured)
+        if (budget > (size_t)maxp * 6 / 10) budget = (size_t)maxp * 6 / 10;
+        if (budget > (size_t)maxw) budget = (size_t)maxw;
+        int k = (int)(budget / layer_bytes);
+        if (p.persist_layers > 0) k = p.persist_layers;  // FT_L2_PERSIST_LAYERS (experiments)
+        if (k > p.D) k = p.D;
+        size_t bytes = (size_t)k * layer_bytes;
+        if (bytes > (size_t)maxw) { k = (int)((size_t)maxw / layer_bytes); bytes = (size_t)k * layer_bytes; }
+        if (k > 0 && maxp > 0 && persisting_limit_at_least(dev, bytes < (size_t)maxp ? bytes : (size_t)maxp, s)) {
+            const size_t lim = bytes < (size_t)maxp ? bytes : (size_t)maxp;
+            q.persist_layers = k;
+            attr2[0] = attr[0];
+            attr2[1].id = cudaLaunchAttributeAccessPolicyWindow;
+            attr2[1].val.accessPolicyWindow.base_ptr = const_cast<void*>(t.W);
+            attr2[1].val.accessPolicyWindow.num_bytes = bytes;
+            attr2[1].val.accessPolicyWindow.hitRatio = (float)lim / (float)bytes;
+            attr2[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+            attr2[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+            cfg.attrs = attr2;
+            cfg.numAttrs = 2;
+        }
     }
-    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, p, t, M);
+    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
 }

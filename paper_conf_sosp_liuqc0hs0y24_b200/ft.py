@@ -25,7 +25,7 @@ FT_MAX_DEPTH = 64
 
 # every symbol include/ft.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = (
-    "ft_version", "ft_status_string", "ft_last_error",
+    "ft_version", "ft_status_string", "ft_last_error", "ft_set_l2_persist",
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
     "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
     "ft_stacked_rnn_workspace_size", "ft_stacked_rnn_fwd",
@@ -56,6 +56,8 @@ def lib():
             raise RuntimeError(f"{LIB_PATH} missing: run `python -m paper_conf_sosp_liuqc0hs0y24_b200.build`")
         L = ctypes.CDLL(LIB_PATH)
         L.ft_version.restype = _c_int
+        L.ft_set_l2_persist.restype = _c_int
+        L.ft_set_l2_persist.argtypes = [_c_int]
         L.ft_status_string.restype = ctypes.c_char_p
         L.ft_status_string.argtypes = [_c_int]
         L.ft_last_error.restype = ctypes.c_char_p
@@ -100,6 +102,11 @@ def lib():
 # ------------------------------------------------------------------------------ raw C ABI
 def ft_version() -> int:
     return lib().ft_version()
+
+
+def ft_set_l2_persist(mib: int) -> int:
+    """Persisting-L2 window size for streaming calls (-1 auto, 0 off, else MiB); returns a status."""
+    return lib().ft_set_l2_persist(mib)
 
 
 def status_string(s: int) -> str:

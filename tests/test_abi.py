@@ -41,6 +41,13 @@ def test_version_and_status_strings():
     assert ft.status_string(42) == "FT_ERR_UNKNOWN"
 
 
+def test_set_l2_persist_validates():
+    assert ft.ft_set_l2_persist(-2) == ft.FT_ERR_INVALID_ARGUMENT
+    assert ft.ft_set_l2_persist(0) == ft.FT_OK
+    assert ft.ft_set_l2_persist(32) == ft.FT_OK
+    assert ft.ft_set_l2_persist(-1) == ft.FT_OK  # back to the default
+
+
 FAKE = 1 << 20  # a 16-byte-aligned non-NULL "device" pointer; never dereferenced on error paths
 
 

@@ -417,3 +417,55 @@ def test_bf16_grid_shapes(B, Lx, Ly, H, D):
     torch.cuda.synchronize()
     ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
     _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n", "h_all", "c_all"), ctx=f"grid {B,Lx,Ly,H,D}")
+
+
+# ------------------------------------------------------------------------- persisting L2 window
+def _streaming_case():
+    # 5 layers x 16 MiB of bf16 weights = 80 MiB: over the 64 MiB L2-resident threshold, so the
+    # call streams its weights and the persisting window applies (W of the first 3 layers at the
+    # default 48 MiB)
+    return ftgen.stacked_inputs(256, 6, 1024, 5, 4242, "bf16")
+
+
+def test_bf16_l2_persist_window_bitwise_and_parity():
+    p = _streaming_case()
+    try:
+        assert ft.ft_set_l2_persist(0) == ft.FT_OK
+        off = _run_stacked(p, torch.bfloat16, want_all=True)
+        assert ft.ft_set_l2_persist(-1) == ft.FT_OK
+        on = _run_stacked(p, torch.bfloat16, want_all=True)
+        assert ft.ft_set_l2_persist(8) == ft.FT_OK  # one layer
+        one = _run_stacked(p, torch.bfloat16, want_all=True)
+    finally:
+        ft.ft_set_l2_persist(-1)
+    for k in ALL:  # the window changes where bytes come from, never the arithmetic
+        assert torch.equal(off[k], on[k]), k
+        assert torch.equal(off[k], one[k]), k
+    rows = [0, 129, 255]
+    _check(on, _oracle_stacked(p, rows=rows), torch.bfloat16, OUT, rows=rows, ctx="persist")
+
+
+def test_bf16_l2_persist_window_under_graph_capture():
+    """A first call made during stream capture must not change the device limit (illegal while
+    capturing); the captured forward still replays to the right answer."""
+    p = _streaming_case()
+    B, T, H, D = 256, 6, 1024, 5
+    x, W, U = (dev(p[k], torch.bfloat16) for k in ("x", "W", "U"))
+    b = dev(p["b"], torch.float32)
+    ws = ft.Workspace()
+    s = torch.cuda.Stream()
+    out = {"y": torch.empty((B, T, H), dtype=torch.bfloat16, device="cuda"),
+           "h_n": torch.empty((B, D, H), dtype=torch.bfloat16, device="cuda"),
+           "c_n": torch.empty((B, D, H), dtype=torch.float32, device="cuda")}
+    with torch.cuda.stream(s):
+        ft.stacked_lstm(x, W, U, b, workspace=ws, out=out, stream=s)
+    s.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        ft.stacked_lstm(x, W, U, b, workspace=ws, out=out, stream=s)
+    for k in out:
+        out[k].zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    rows = [1, 200]
+    _check(out, _oracle_stacked(p, rows=rows), torch.bfloat16, OUT, rows=rows, ctx="persist graph")
