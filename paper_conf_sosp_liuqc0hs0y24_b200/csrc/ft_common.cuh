@@ -41,8 +41,9 @@ struct Problem {
     int persist_layers;  // bf16 streaming: W of the first persist_layers layers lie in a persisting
                          // L2 access-policy window (loaded with EVICT_NORMAL); host side: -1 = auto
     int debug;           // timing experiments only (env FT_DEBUG; results invalid when != 0):
-                         // bit 0 skip dependency waits, bit 1 skip the epilogue math/stores;
-                         // bit 6 (64) = stress mode: random delays before each counter release
+                         // 1 skip dependency waits, 2 skip the epilogue math/stores, 4 no MMAs,
+                         // 16 no weight loads, 32 fixed load coordinates, 128 EVICT_NORMAL state;
+                         // 64 = stress mode: random delays before each counter release
                          // (results stay valid; used by tests to shake out ordering bugs)
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT

@@ -197,8 +197,8 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const uint64_t pol_stream = policy_evict_first();
     const uint64_t pol_keep = policy_evict_last();
     const uint64_t pol_act = policy_evict_normal();
-    const bool skipA = P.debug & 8, skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
-    const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : (skipA ? 0 : CG * C::A_BYTES);
+    const bool skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
+    const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : CG * C::A_BYTES;
     const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
     FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
@@ -214,14 +214,6 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
         if constexpr (!kWeights) {
             FT_TR_ADD(TR_TILES, 1);
             if (rank == 0) FT_EV(tile, 0);
-            if (P.debug & 256) {  // A/B experiment: acquire every producer before any load
-                long long prod[3];
-                producers(P, tl.cell, prod);
-#pragma unroll
-                for (int q = 0; q < 3; ++q)
-                    if (prod[q] >= 0) wait_flag_geq(T.flags + prod[q] * P.MB + tl.m, target);
-                fence_proxy_async_global();
-            }
         }
         int si = 0, kc = 0;
         for (int c = 0; c < nchunks; ++c) {
@@ -255,7 +247,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                                               fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
                 }
             } else {
-                if (!skipA) load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
+                load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
             }
             if (++kc == kchunks) { kc = 0; si = next_segment(seg, si); }
             if (++stage == C::STAGES) {
@@ -569,13 +561,6 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 bg[v] = t3.x; bg[v + 1] = t3.y; bg[v + 2] = t3.z; bg[v + 3] = t3.w;
             }
             float hv[16];
-            if (P.debug & 1024) {  // timing experiment: no gate math (wrong results)
-#pragma unroll
-                for (int v = 0; v < 16; ++v) {
-                    cv[u0 + v] = zf[v] + cp[u0 + v];
-                    hv[v] = zi[v] + zo[v] + zg[v];
-                }
-            } else
 #pragma unroll
             for (int v = 0; v < 16; ++v) {
                 const float ig = sigmoid_approx(zi[v] + bi[v]);
@@ -594,15 +579,15 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                                             pack_bf16x2(hv[8 * w + 6], hv[8 * w + 7]));
             // what downstream cells read — h (blocked SSA buffer hb) and c (ring) — stored per
             // chunk so the stores overlap the next chunk's math
-            if (valid && !(P.debug & 512)) {  // bits 512 / 2048 / 4096: timing experiments (no h/c, c, h stores)
+            if (valid) {
                 const int nn = n0 + u0;
                 uint4* hdst = reinterpret_cast<uint4*>(
                     (__nv_bfloat16*)T.hb + hb_row(P, row_h, nn / 64, b) * 64 + (nn % 64));
-                if (!(P.debug & 4096)) st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
+                st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
                 float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn);
 #pragma unroll
                 for (int v = 0; v < 4; ++v)
-                    if (!(P.debug & 2048)) st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
+                    st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
                                make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
                                           __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
                                pol_state);
