@@ -23,6 +23,7 @@ run_seq(130, 4, 128, 2, torch.bfloat16)               # streaming, CTA pair
 run_seq(20, 7, 128, 3, torch.bfloat16, dil=[1, 2, 3])
 run_grid(3, 3, 4, 64, 2, torch.bfloat16)
 run_grid(3, 3, 4, 16, 2, torch.float32)
+run_seq(256, 2, 1024, 5, torch.bfloat16, resident="0")  # streaming weights (80 MiB): persisting L2 window
 os.environ["FT_TILE_UNITS"] = "32"
 run_seq(130, 4, 128, 2, torch.bfloat16, resident="0")  # CTA pair, 32-unit tiles
 os.environ.pop("FT_TILE_UNITS")
