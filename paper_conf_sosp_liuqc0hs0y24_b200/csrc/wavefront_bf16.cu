@@ -427,10 +427,8 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
             ydst[1] = hp[1];
         }
         named_bar_sync(1, EPI_THREADS);
-        if (leader_thread) {
-            __threadfence();
+        if (leader_thread)  // one cumulative release after the barrier (as in run_epilogue)
             red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
-        }
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }

@@ -54,6 +54,12 @@ __device__ __forceinline__ uint32_t pack2(float lo, float hi) {
     return *reinterpret_cast<uint32_t*>(&v);
 }
 
+// shared-memory layout: weight slab | A ring | barriers + TMEM slot (256 B) | bias [4][BNUR]
+template <int BNUR>
+__host__ __device__ constexpr int resident_bias_off(int H) {
+    return 2 * (H / RBK) * RCfg<BNUR>::WCHUNK + RCfg<BNUR>::STAGES * RCfg<BNUR>::A_BYTES + 256;
+}
+
 template <int BNUR>
 __global__ void __launch_bounds__(RTHREADS, 1)
 wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
@@ -72,6 +78,7 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
     uint64_t* tempty = tfull + 2;
     uint64_t* wbar = tempty + 2;
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
+    float* sbias = reinterpret_cast<float*>(smem_raw + pad + resident_bias_off<BNUR>(P.H));  // [4][BNUR]
 
     const int NTR = P.H / BNUR;
     const int d = blockIdx.x / NTR, n = blockIdx.x % NTR;
@@ -89,6 +96,13 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
         fence_mbarrier_init();
     }
     if (warp == 1) tmem_alloc(tmem_slot, C::TMEM_COLS);
+    // the slab's bias → shared memory once: the per-step acquires invalidate L1 (CCTL.IVALL), so
+    // global bias loads in the epilogue would go to L2 on the critical path every step
+    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * BNUR) {
+        const int e = threadIdx.x - 64;
+        sbias[e] = T.b[(long long)(blockIdx.x / (P.H / BNUR)) * 4 * P.H + (e / BNUR) * P.H +
+                       (blockIdx.x % (P.H / BNUR)) * BNUR + e % BNUR];
+    }
     tc_fence_before();
     __syncthreads();
     tc_fence_after();
@@ -184,7 +198,6 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
         const int q = warp & 3, row = q * 32 + lane;
         const bool valid = row < P.B;
         const int n0 = n * BNUR;
-        const float* bias = T.b + (long long)d * 4 * P.H + n0;
         float creg[BNUR];
 #pragma unroll
         for (int u = 0; u < BNUR; ++u) creg[u] = 0.f;
@@ -212,10 +225,10 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
                 }
 #pragma unroll
                 for (int v = 0; v < 16; ++v) {
-                    const float ig = sigmoid_approx(zi[v] + __ldg(bias + 0 * P.H + u0 + v));
-                    const float fg = sigmoid_approx(zf[v] + __ldg(bias + 1 * P.H + u0 + v));
-                    const float og = sigmoid_approx(zo[v] + __ldg(bias + 2 * P.H + u0 + v));
-                    const float gh = tanh_approx(zg[v] + __ldg(bias + 3 * P.H + u0 + v));
+                    const float ig = sigmoid_approx(zi[v] + sbias[0 * BNUR + u0 + v]);
+                    const float fg = sigmoid_approx(zf[v] + sbias[1 * BNUR + u0 + v]);
+                    const float og = sigmoid_approx(zo[v] + sbias[2 * BNUR + u0 + v]);
+                    const float gh = tanh_approx(zg[v] + sbias[3 * BNUR + u0 + v]);
                     creg[u0 + v] = fmaf(fg, creg[u0 + v], ig * gh);
                     zi[v] = og * tanh_approx(creg[u0 + v]);  // h
                 }
@@ -229,11 +242,8 @@ wavefront_resident_kernel(const __grid_constant__ Problem P, const __grid_consta
                 for (int w = 0; w < BNUR / 8; ++w)
                     __stcg(dst + w, make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]));
             }
-            named_bar_sync(1, 128);
-            if (threadIdx.x == 64) {
-                __threadfence();
-                red_release_gpu_add(T.flags + cell_lin(P, d, t, 0), 1);
-            }
+            named_bar_sync(1, 128);  // every epilogue thread's h stores, then ONE cumulative release
+            if (threadIdx.x == 64) red_release_gpu_add(T.flags + cell_lin(P, d, t, 0), 1);
             if (valid) {  // outputs nobody inside the nest reads
                 const long long hi = h_all_index(P, cell, 0, row, n0);
                 if (h_all) {
@@ -299,7 +309,7 @@ bool enc_map(EncodeTiledFn enc, CUtensorMap* m, int rank, const void* base, cons
 template <int BNUR>
 size_t resident_smem(int H) {
     using C = RCfg<BNUR>;
-    return (size_t)2 * (H / RBK) * C::WCHUNK + C::STAGES * C::A_BYTES + 256 + 1024;
+    return (size_t)2 * (H / RBK) * C::WCHUNK + C::STAGES * C::A_BYTES + 256 + 4 * BNUR * 4 + 1024;
 }
 
 template <int BNUR>
