@@ -45,6 +45,8 @@ cudaError_t launch_b2b_gemm(int M, int N, const void* A, const void* B, const vo
                             cudaStream_t s, std::string* err);
 // a5 weight-resident mode (wavefront_resident.cu): slab width 16/32 when the weights fit, else 0
 int resident_bnu(const Problem& p, int nsm);
+bool cluster_kernel_applies(const Problem& p);
+cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err);
 cudaError_t launch_wavefront_resident(const Problem& p, const Tensors& t, cudaStream_t s, int bnu,
                                       std::string* err);
 

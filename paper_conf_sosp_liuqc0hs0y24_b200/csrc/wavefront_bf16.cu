@@ -965,8 +965,13 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned l
 
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
                                   std::string* err) {
-    // a5: weights resident in shared memory for the whole sequence when they fit
+    // latency-bound small stacked LSTMs (C2): weights resident in the SMEM of one cluster per
+    // layer, h exchanged through DSMEM on the time edge (wavefront_cluster.cu)
+    const char* envc = getenv("FT_CLUSTER");  // "0" disables it (comparisons)
     const char* env = getenv("FT_RESIDENT");  // "0" forces the streaming kernel (comparisons)
+    if (!(envc && envc[0] == '0') && !(env && env[0] == '0') && cluster_kernel_applies(p))
+        return launch_wavefront_cluster(p, t, s, err);
+    // a5: weights resident in shared memory for the whole sequence when they fit
     if (p.BM == ROWS && !(env && env[0] == '0')) {
         int dev = 0, nsm = 0;
         if (cudaGetDevice(&dev) == cudaSuccess &&

@@ -1,0 +1,496 @@
+// wavefront_cluster.cu — the latency-bound stacked LSTM (e.g. C2) with the recurrent state
+// exchanged through distributed shared memory.
+//
+// In a wavefront every monotone path from cell (0, 0) to (D-1, T-1) has exactly T-1 time edges
+// (h_{d,t-1} → cell (d, t), Listing 2) and D-1 depth edges (h_{d-1,t} → cell (d, t),
+// Listing 1), so the critical path is (T-1)·latency(time edge) + (D-1)·latency(depth
+// edge) (Table 4 dependence vectors, L307–L317).  With T ≫ D the time edge dominates.  Here one
+// layer's hidden units are split over a thread-block cluster (H/32 CTAs, 32 units each) whose
+// CTAs keep their weight slab resident in shared memory (the reuse of L345–L349, as in
+// wavefront_resident.cu) and hand h_{d,t} to each other through DSMEM: every CTA stages its
+// 32-unit slice of h_{d,t} in shared memory and bulk-copies it (cp.async.bulk shared::cluster,
+// complete_tx on the receiver's mbarrier) into every cluster CTA's recurrent operand buffer.  The
+// receiver's MMA warp waits on that mbarrier — no global-memory round trip, no readiness counter
+// on the time edge.  Depth edges (layer d-1 → d, another cluster) still go through the blocked
+// SSA buffer hb + a release/acquire counter, as in the other kernels.
+//
+// Shapes: batch B <= 64 (the tile is M = 128 with rows >= B never stored), H in {128, 256}
+// (cluster of H/32 <= 8 CTAs), stacked (dilation 1).  N = 4 gates x 32 units = 128, K = 64 per
+// chunk.  Warps: 0 TMA producer, 1 MMA issuer (whole warp), 2–5 epilogue (warps of TMEM lane
+// quadrants 0 and 1, i.e. rows 0..63, do the work).
+//
+// Recurrent operand layout (no swizzle, K-major): k-group g (8 units, 16 bytes) of all 64 rows is
+// one contiguous 1 KiB block (row r at r*16), so CTA j's 32 units = k-groups 4j..4j+3 = ONE
+// contiguous 4 KiB run in every receiver.  UMMA descriptor: core matrix = 8 rows x 16 B
+// (128 contiguous bytes), LBO = 1 KiB (next core matrix along K), SBO = 128 B (next 8 rows).
+// Rows 64..127 of the M = 128 operand read the next k-group's block (or the following buffer):
+// garbage rows whose accumulator lanes are never read.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <string>
+
+#include "ft_internal.h"
+#include "ft_sm100.cuh"
+
+namespace ft {
+
+#ifdef FT_TRACE
+// development-only (libft_trace.so): per-step %globaltimer stamps of CTA `g_cev_cta`:
+// 0 MMA warp saw hfull, 1 MMA warp committed, 2 epilogue saw tfull, 3 math done, 4 copies issued,
+// 5 x-half ready (MMA warp saw the first xfull of the step)
+__device__ unsigned long long g_cev[4096 * 8];
+__device__ int g_cev_cta = 0;
+#define FT_CEV(t, k) do { if (blockIdx.x == g_cev_cta && (t) < 4096) g_cev[(t) * 8 + (k)] = globaltimer_ns(); } while (0)
+extern "C" __attribute__((visibility("default"))) int ft_debug_cluster_events(unsigned long long* host, int nsteps, int cta) {
+    if (nsteps > 4096) nsteps = 4096;
+    cudaDeviceSynchronize();
+    if (cudaMemcpyFromSymbol(host, g_cev, (size_t)nsteps * 8 * 8) != cudaSuccess) return -1;
+    cudaMemcpyToSymbol(g_cev_cta, &cta, sizeof(int));
+    return nsteps;
+}
+#else
+#define FT_CEV(t, k) ((void)0)
+#endif
+
+namespace {
+
+using namespace sm100;
+
+constexpr int KROWS = 128;  // UMMA M
+constexpr int KB = 64;      // batch rows actually carried (B <= KB)
+constexpr int KU = 32;      // hidden units per CTA
+constexpr int KN = 4 * KU;  // UMMA N (i | f | o | ĝ)
+constexpr int KBK = 64;     // K per chunk
+constexpr int KTHREADS = 192;
+constexpr int XSTAGES = 3;
+constexpr int X_BYTES = KB * KBK * 2;          // 8 KiB: 64 rows x 64 units (SW128)
+constexpr int GATE_BYTES = KU * KBK * 2;       // 4 KiB: one gate's 32 units x 64 K (SW64)
+constexpr int WCHUNK = 4 * GATE_BYTES;         // 16 KiB
+constexpr int SLICE_BYTES = KB * KU * 2;       // 4 KiB: one CTA's h slice (4 k-groups x 64 rows)
+constexpr uint32_t IDESC = make_idesc_bf16_f32(KROWS, KN, false, true);
+
+struct KMaps {
+    CUtensorMap x, h, W, U;
+};
+
+struct KLayout {  // byte offsets into the 1024-aligned dynamic shared memory
+    int rec0, rec1, xring, w, stage, bars, bias, total;
+};
+
+__host__ __device__ constexpr KLayout klayout(int H) {
+    KLayout L{};
+    const int rec = (H / 8) * 1024;  // H/8 k-groups x 1 KiB
+    L.rec0 = 0;
+    L.rec1 = rec;
+    L.xring = 2 * rec;
+    L.w = L.xring + XSTAGES * X_BYTES;
+    L.stage = L.w + 2 * (H / KBK) * WCHUNK;
+    L.bars = L.stage + SLICE_BYTES;
+    L.bias = L.bars + 256;
+    L.total = L.bias + 4 * KU * 4;
+    return L;
+}
+
+__device__ __forceinline__ uint32_t kpack(float lo, float hi) {
+    __nv_bfloat162 v = __floats2bfloat162_rn(lo, hi);
+    return *reinterpret_cast<uint32_t*>(&v);
+}
+
+// Bulk copy of `bytes` from this CTA's shared memory into a cluster peer's shared memory; the
+// peer's mbarrier receives complete_tx(bytes).
+__device__ __forceinline__ void bulk_s2cluster(uint32_t dst_cluster, uint32_t src_cta, uint32_t bytes,
+                                               uint32_t mbar_cluster) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            dst_cluster),
+        "r"(src_cta), "r"(bytes), "r"(mbar_cluster)
+        : "memory");
+}
+__device__ __forceinline__ void bulk_commit_and_wait_read() {
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+
+__global__ void __launch_bounds__(KTHREADS, 1)
+wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
+                         const __grid_constant__ KMaps M) {
+    extern __shared__ uint8_t smem_raw[];
+    const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
+    uint8_t* smem = smem_raw + pad;
+    const KLayout L = klayout(P.H);
+    const int KCH = P.H / KBK;           // K chunks per half
+    const int CS = P.H / KU;             // CTAs per layer = cluster size
+    uint8_t* rec[2] = {smem + L.rec0, smem + L.rec1};
+    uint8_t* xring = smem + L.xring;
+    uint8_t* sW = smem + L.w;
+    uint8_t* stage_buf = smem + L.stage;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
+    uint64_t* xfull = bars;                       // [XSTAGES]
+    uint64_t* xempty = bars + XSTAGES;            // [XSTAGES]
+    uint64_t* tfull = bars + 2 * XSTAGES;         // [2]
+    uint64_t* tempty = tfull + 2;                 // [2]
+    uint64_t* hfull = tempty + 2;                 // [2] recurrent buffers (DSMEM complete_tx)
+    uint64_t* wbar = hfull + 2;
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(wbar + 1);
+    float* sbias = reinterpret_cast<float*>(smem + L.bias);  // [4][KU]
+
+    const uint32_t j = cluster_ctarank();        // unit slab inside the layer
+    const int d = blockIdx.x / CS;               // layer = cluster
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rec_bytes = (uint32_t)KB * P.H * 2;  // one full h_{d,t} (all CS slices)
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < XSTAGES; ++s) {
+            mbar_init(&xfull[s], 1);
+            mbar_init(&xempty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull[a], 1);
+            mbar_init(&tempty[a], 2);  // the two working epilogue warps
+            mbar_init(&hfull[a], 1);
+        }
+        mbar_init(wbar, 1);
+        fence_mbarrier_init();
+        // arm both recurrent buffers for their first phase (h_0 → rec0, h_1 → rec1) before any
+        // peer can send: the cluster barrier below orders this before every peer's first copy
+        mbar_arrive_expect_tx(&hfull[0], rec_bytes);
+        mbar_arrive_expect_tx(&hfull[1], rec_bytes);
+    }
+    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * KU) {
+        const int e = threadIdx.x - 64;
+        sbias[e] = T.b[(long long)d * 4 * P.H + (e / KU) * P.H + (int)j * KU + e % KU];
+    }
+    if (warp == 1) tmem_alloc(tmem_slot, 2 * KN);
+    tc_fence_before();
+    __syncthreads();
+    cluster_sync();
+    tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+
+    if (warp == 0) {
+        if (lane == 0) {
+            // ---- the slab's weights → shared memory, once for the whole sequence -------------
+            const uint64_t pol_keep = policy_evict_last();
+            const uint64_t pol_act = policy_evict_normal();
+            mbar_arrive_expect_tx(wbar, 2 * KCH * WCHUNK);
+            for (int c = 0; c < 2 * KCH; ++c)
+                tma_load_4d_hint_addr<1>(smem_u32(sW + c * WCHUNK), c < KCH ? &M.W : &M.U, smem_u32(wbar),
+                                         (int)j * KU, (c % KCH) * KBK, 0, d, pol_keep);
+            // ---- per step: the input half (x or the layer below) -----------------------------
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int t = 0; t < P.L0; ++t) {
+                if (d > 0) {  // depth edge: layer d-1's cell (d-1, t), all CS slices
+                    wait_flag_geq(T.flags + cell_lin(P, d - 1, t, 0), CS);
+                    fence_proxy_async_global();
+                }
+                for (int kc = 0; kc < KCH; ++kc) {
+                    mbar_wait(&xempty[stage], phase ^ 1);
+                    mbar_arrive_expect_tx(&xfull[stage], X_BYTES);
+                    const uint32_t dst = smem_u32(xring + stage * X_BYTES);
+                    const uint32_t bar = smem_u32(&xfull[stage]);
+                    if (d == 0)
+                        tma_load_3d_hint_addr<1>(dst, &M.x, bar, kc * KBK, t, 0, pol_act);
+                    else
+                        tma_load_2d_hint_addr<1>(dst, &M.h, bar, 0,
+                                                 (int)hb_row(P, h_row(P, d - 1, t, 0, 0), kc, 0), pol_act);
+                    if (++stage == XSTAGES) {
+                        stage = 0;
+                        phase ^= 1;
+                    }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ---- MMA issuer (whole warp; warp-uniform waits keep descriptors uniform) ------------
+        mbar_wait_warp(wbar, 0);
+        tc_fence_after();
+        const uint64_t xdesc0 = make_sdesc(smem_u32(xring), 16, 1024);                 // SW128 K-major
+        const uint64_t rdesc[2] = {make_sdesc(smem_u32(rec[0]), 1024, 128, 0),         // no swizzle
+                                   make_sdesc(smem_u32(rec[1]), 1024, 128, 0)};
+        const uint64_t bdesc0 = make_sdesc(smem_u32(sW), GATE_BYTES, 8 * KU * 2, 4u);   // SW64 MN-major
+        int stage = 0, acc = 0;
+        uint32_t phase = 0, acc_phase = 0;
+        for (int t = 0; t < P.L0; ++t) {
+            mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
+            tc_fence_after();
+            const uint32_t d_tmem = tmem_base + (uint32_t)(acc * KN);
+            // input half first: it arrives early (the layer below runs ahead)
+            for (int kc = 0; kc < KCH; ++kc) {
+                mbar_wait_warp(&xfull[stage], phase);
+                if (kc == 0 && lane == 0) FT_CEV(t, 5);
+                tc_fence_after();
+                if (elect_one()) {
+                    const uint64_t ad = xdesc0 + (uint64_t)((stage * X_BYTES) >> 4);
+                    const uint64_t bd = bdesc0 + (uint64_t)((kc * WCHUNK) >> 4);
+#pragma unroll
+                    for (int kk = 0; kk < KBK / 16; ++kk)
+                        umma_f16(d_tmem, ad + (uint64_t)((kk * 32) >> 4), bd + (uint64_t)((kk * 16 * KU * 2) >> 4),
+                                 IDESC, (kc | kk) != 0);
+                    umma_commit(&xempty[stage]);
+                }
+                __syncwarp();
+                if (++stage == XSTAGES) {
+                    stage = 0;
+                    phase ^= 1;
+                }
+            }
+            if (t > 0) {  // time edge: h_{d,t-1} from every cluster CTA, through DSMEM
+                const int p = (t - 1) & 1;
+                mbar_wait_warp(&hfull[p], (uint32_t)((t - 1) >> 1) & 1u);
+                if (lane == 0) FT_CEV(t, 0);
+                tc_fence_after();
+                if (elect_one()) {
+                    // re-arm this buffer for h_{t+1}: its senders first need our h_t, which we
+                    // send only after these MMAs completed — so the next phase cannot start early
+                    mbar_arrive_expect_tx(&hfull[p], rec_bytes);
+                    for (int kc = 0; kc < KCH; ++kc) {
+                        const uint64_t bd = bdesc0 + (uint64_t)(((KCH + kc) * WCHUNK) >> 4);
+#pragma unroll
+                        for (int kk = 0; kk < KBK / 16; ++kk)
+                            umma_f16(d_tmem, rdesc[p] + (uint64_t)(((kc * 8 + kk * 2) * 1024) >> 4),
+                                     bd + (uint64_t)((kk * 16 * KU * 2) >> 4), IDESC, 1u);
+                    }
+                }
+                __syncwarp();
+            }
+            if (elect_one()) umma_commit(&tfull[acc]);
+            if (lane == 0) FT_CEV(t, 1);
+            __syncwarp();
+            acc ^= 1;
+            if (acc == 0) acc_phase ^= 1;
+        }
+    } else if ((warp & 3) < 2) {
+        // ---- epilogue: warps of TMEM lane quadrants 0 and 1 (rows 0..63); c in registers ------
+        const int q = warp & 3, row = q * 32 + lane;
+        const bool valid = row < P.B;
+        const int n0 = (int)j * KU;
+        const bool sender = (warp == 4 && lane == 0);
+        float creg[KU];
+#pragma unroll
+        for (int u = 0; u < KU; ++u) creg[u] = 0.f;
+        __nv_bfloat16* hb = (__nv_bfloat16*)T.hb;
+        __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
+        int acc = 0;
+        uint32_t acc_phase = 0;
+        for (int t = 0; t < P.L0; ++t) {
+            mbar_wait(&tfull[acc], acc_phase);
+            if (sender) FT_CEV(t, 2);
+            tc_fence_after();
+            const uint32_t tbase = tmem_base + (uint32_t)(acc * KN) + ((uint32_t)(q * 32) << 16);
+            uint32_t hp[KU / 2];
+#pragma unroll
+            for (int u0 = 0; u0 < KU; u0 += 16) {
+                float zi[16], zf[16], zo[16], zg[16];
+                tmem_ld_32x32b_x16(tbase + 0 * KU + u0, zi);
+                tmem_ld_32x32b_x16(tbase + 1 * KU + u0, zf);
+                tmem_ld_32x32b_x16(tbase + 2 * KU + u0, zo);
+                tmem_ld_32x32b_x16(tbase + 3 * KU + u0, zg);
+                tmem_wait_ld();
+                if (u0 + 16 == KU) {
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive(&tempty[acc]);
+                }
+#pragma unroll
+                for (int v = 0; v < 16; ++v) {
+                    const float ig = sigmoid_approx(zi[v] + sbias[0 * KU + u0 + v]);
+                    const float fg = sigmoid_approx(zf[v] + sbias[1 * KU + u0 + v]);
+                    const float og = sigmoid_approx(zo[v] + sbias[2 * KU + u0 + v]);
+                    const float gh = tanh_approx(zg[v] + sbias[3 * KU + u0 + v]);
+                    creg[u0 + v] = fmaf(fg, creg[u0 + v], ig * gh);
+                    zi[v] = og * tanh_approx(creg[u0 + v]);  // h
+                }
+#pragma unroll
+                for (int v = 0; v < 8; ++v) hp[u0 / 2 + v] = kpack(zi[2 * v], zi[2 * v + 1]);
+            }
+            // (1) the time edge first: stage the slice (k-group-major, row r at r*16 in each
+            //     1 KiB k-group block) and bulk-copy it into every cluster CTA's buffer t & 1
+            if (sender) FT_CEV(t, 3);
+            if (t + 1 < P.L0) {
+                if (sender) bulk_commit_and_wait_read();  // the previous step's copies read the stage
+                named_bar_sync(1, 64);
+#pragma unroll
+                for (int g = 0; g < KU / 8; ++g)
+                    *reinterpret_cast<uint4*>(stage_buf + g * 1024 + row * 16) =
+                        make_uint4(hp[4 * g], hp[4 * g + 1], hp[4 * g + 2], hp[4 * g + 3]);
+                fence_proxy_async_smem();  // generic-proxy writes → the bulk copy's async-proxy reads
+                named_bar_sync(1, 64);
+                if (sender) {
+                    const uint32_t src = smem_u32(stage_buf);
+                    const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES;
+                    const uint32_t bar_local = smem_u32(&hfull[t & 1]);
+                    for (int r = 0; r < CS; ++r)
+                        bulk_s2cluster(mapa_shared(dst_local, (uint32_t)r), src, SLICE_BYTES,
+                                       mapa_shared(bar_local, (uint32_t)r));
+                    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+                    FT_CEV(t, 4);
+                }
+            }
+            // (2) the depth edge: h into the blocked SSA buffer, then one cumulative release
+            const Cell cell{d + t, d, t, 0};
+            if (valid) {
+                uint4* dst = reinterpret_cast<uint4*>(hb + hb_row(P, h_row(P, d, t, 0, 0), n0 / 64, row) * 64 + (n0 % 64));
+#pragma unroll
+                for (int w = 0; w < KU / 8; ++w)
+                    __stcg(dst + w, make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]));
+            }
+            named_bar_sync(1, 64);
+            if (sender && d + 1 < P.D) red_release_gpu_add(T.flags + cell_lin(P, d, t, 0), 1);
+            // (3) outputs nobody inside the nest reads
+            if (valid) {
+                const long long hi = h_all_index(P, cell, 0, row, n0);
+                if (h_all) {
+                    uint4* dh = reinterpret_cast<uint4*>(h_all + hi);
+#pragma unroll
+                    for (int w = 0; w < KU / 8; ++w)
+                        dh[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
+                }
+                if (T.c_all) {
+                    float4* dc = reinterpret_cast<float4*>(T.c_all + hi);
+#pragma unroll
+                    for (int w = 0; w < KU / 4; ++w)
+                        dc[w] = make_float4(creg[4 * w], creg[4 * w + 1], creg[4 * w + 2], creg[4 * w + 3]);
+                }
+                if (d == P.D - 1) {
+                    uint4* dy = reinterpret_cast<uint4*>((__nv_bfloat16*)T.y + y_index(P, cell, 0, row, n0));
+#pragma unroll
+                    for (int w = 0; w < KU / 8; ++w)
+                        dy[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
+                }
+                if (t == P.L0 - 1) {
+                    const long long ni = hn_index(P, cell, 0, row, n0);
+                    uint4* dn = reinterpret_cast<uint4*>((__nv_bfloat16*)T.h_n + ni);
+#pragma unroll
+                    for (int w = 0; w < KU / 8; ++w)
+                        dn[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
+                    float4* dc = reinterpret_cast<float4*>(T.c_n + ni);
+#pragma unroll
+                    for (int w = 0; w < KU / 4; ++w)
+                        dc[w] = make_float4(creg[4 * w], creg[4 * w + 1], creg[4 * w + 2], creg[4 * w + 3]);
+                }
+            }
+            acc ^= 1;
+            if (acc == 0) acc_phase ^= 1;
+        }
+        if (sender) bulk_commit_and_wait_read();
+    }
+    tc_fence_before();
+    __syncthreads();
+    cluster_sync();  // no CTA leaves while a peer may still copy into its shared memory
+    if (warp == 1) {
+        tc_fence_after();
+        tmem_dealloc(tmem_base, 2 * KN);
+    }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+bool kenc(EncodeTiledFn enc, CUtensorMap* m, int rank, const void* base, const cuuint64_t* dims,
+          const cuuint64_t* strides, const cuuint32_t* box, CUtensorMapSwizzle sw, std::string* err) {
+    const cuuint32_t es[4] = {1, 1, 1, 1};
+    CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, rank, const_cast<void*>(base), dims, strides, box, es,
+                     CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS) {
+        if (err) *err = "cuTensorMapEncodeTiled (cluster) failed: " + std::to_string((int)r);
+        return false;
+    }
+    return true;
+}
+
+size_t cluster_smem(int H) { return (size_t)klayout(H).total + 1024; }
+
+}  // namespace
+
+// The DSMEM-exchange kernel applies when: stacked LSTM (every dilation 1), batch <= 64, H in
+// {128, 256}, bf16, and the D clusters of H/32 CTAs (one CTA per SM) can all be co-resident.
+bool cluster_kernel_applies(const Problem& p) {
+    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM || p.B > KB || (p.H != 128 && p.H != 256)) return false;
+    for (int d = 0; d < p.D; ++d)
+        if (p.dil[d] != 1) return false;
+    if (cluster_smem(p.H) > 227 * 1024) return false;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return false;
+    cudaFuncSetAttribute(wavefront_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cluster_smem(p.H));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(p.D * (p.H / KU)));
+    cfg.blockDim = dim3(KTHREADS);
+    cfg.dynamicSmemBytes = cluster_smem(p.H);
+    cudaLaunchAttribute a[1];
+    a[0].id = cudaLaunchAttributeClusterDimension;
+    a[0].val.clusterDim.x = p.H / KU;
+    a[0].val.clusterDim.y = 1;
+    a[0].val.clusterDim.z = 1;
+    cfg.attrs = a;
+    cfg.numAttrs = 1;
+    int n = 0;
+    if (cudaOccupancyMaxActiveClusters(&n, wavefront_cluster_kernel, &cfg) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    return n >= p.D;
+}
+
+cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+    void* ptr = nullptr;
+    cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
+    cudaError_t e = cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &ptr, 12000, cudaEnableDefault, &q);
+    if (e != cudaSuccess || !ptr) {
+        if (err) *err = "cuTensorMapEncodeTiled not available";
+        return cudaErrorNotSupported;
+    }
+    EncodeTiledFn enc = reinterpret_cast<EncodeTiledFn>(ptr);
+    KMaps M;
+    const int H = p.H;
+    {  // x [B][T][H]: a (64 units, 1 step, 64 rows) box
+        const cuuint64_t dims[3] = {(cuuint64_t)H, (cuuint64_t)p.L0, (cuuint64_t)p.B};
+        const cuuint64_t st[2] = {(cuuint64_t)H * 2, (cuuint64_t)p.L0 * H * 2};
+        const cuuint32_t box[3] = {KBK, 1, KB};
+        if (!kenc(enc, &M.x, 3, t.x, dims, st, box, CU_TENSOR_MAP_SWIZZLE_128B, err)) return cudaErrorInvalidValue;
+    }
+    {  // blocked SSA buffer hb: a (64 units, 64 rows) box
+        const cuuint64_t dims[2] = {64, (cuuint64_t)hb_rows_total(p)};
+        const cuuint64_t st[1] = {128};
+        const cuuint32_t box[2] = {KBK, KB};
+        if (!kenc(enc, &M.h, 2, t.hb, dims, st, box, CU_TENSOR_MAP_SWIZZLE_128B, err)) return cudaErrorInvalidValue;
+    }
+    {  // weights (n, k, gate, layer): (32 units, 64 K, 4 gates, 1) boxes, 64-byte swizzle
+        const cuuint64_t dims[4] = {(cuuint64_t)H, (cuuint64_t)H, 4, (cuuint64_t)p.D};
+        const cuuint64_t st[3] = {(cuuint64_t)H * 2, (cuuint64_t)H * H * 2, (cuuint64_t)4 * H * H * 2};
+        const cuuint32_t box[4] = {KU, KBK, 4, 1};
+        if (!kenc(enc, &M.W, 4, t.W, dims, st, box, CU_TENSOR_MAP_SWIZZLE_64B, err)) return cudaErrorInvalidValue;
+        if (!kenc(enc, &M.U, 4, t.U, dims, st, box, CU_TENSOR_MAP_SWIZZLE_64B, err)) return cudaErrorInvalidValue;
+    }
+    const size_t smem = cluster_smem(H);
+    e = cudaFuncSetAttribute(wavefront_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) {
+        if (err) *err = std::string("cluster launch setup: ") + cudaGetErrorString(e);
+        return e;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(p.D * (H / KU)));
+    cfg.blockDim = dim3(KTHREADS);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;  // one cluster per layer
+    attr[0].val.clusterDim.x = H / KU;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, wavefront_cluster_kernel, p, t, M);
+    if (e != cudaSuccess && err) *err = std::string("cluster launch: ") + cudaGetErrorString(e);
+    return e;
+}
+
+}  // namespace ft

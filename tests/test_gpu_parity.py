@@ -132,9 +132,36 @@ def test_bf16_resident_vs_streaming(mode, B, T, H, D, monkeypatch):
     """a5: the weight-resident kernel (weights in SMEM for the whole sequence, c in registers)
     and the streaming kernel both match the oracle on shapes where the weights fit."""
     monkeypatch.setenv("FT_RESIDENT", "1" if mode == "resident" else "0")
+    monkeypatch.setenv("FT_CLUSTER", "0")  # the DSMEM cluster kernel has its own tests below
     p = ftgen.stacked_inputs(B, T, H, D, 707 + H, "bf16")
     got = _run_stacked(p, torch.bfloat16, want_all=True)
     _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"{mode} {B,T,H,D}")
+
+
+@pytest.mark.parametrize("B,T,H,D", [(64, 9, 256, 8), (1, 1, 128, 1), (1, 2, 256, 1), (37, 5, 128, 3),
+                                     (64, 3, 256, 2), (17, 12, 256, 5), (64, 33, 128, 4)])
+def test_bf16_cluster_dsmem(B, T, H, D, monkeypatch):
+    """The DSMEM-exchange kernel (one cluster per layer, h_{d,t} bulk-copied into every cluster
+    CTA's recurrent operand buffer): parity with the oracle, and bitwise agreement with the
+    weight-resident kernel is NOT expected (different tile shapes), so both are checked against
+    the oracle; ragged batch (rows >= B are garbage rows of the M = 128 tile), T = 1 (no time
+    edge), one layer (no depth edge), odd lengths (both recurrent buffers and phases)."""
+    monkeypatch.setenv("FT_CLUSTER", "1")
+    p = ftgen.stacked_inputs(B, T, H, D, 909 + B + T, "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"cluster {B,T,H,D}")
+
+
+def test_bf16_cluster_stress_and_repeat(monkeypatch):
+    """Random release delays on the depth edge (stress mode) and repeated calls on one workspace:
+    results bitwise identical run to run."""
+    monkeypatch.setenv("FT_CLUSTER", "1")
+    p = ftgen.stacked_inputs(48, 20, 256, 6, 4711, "bf16")
+    a = _run_stacked(p, torch.bfloat16, want_all=True)
+    b = _run_stacked(p, torch.bfloat16, want_all=True)
+    for k in ALL:
+        assert torch.equal(a[k], b[k]), k
+    _check(a, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="cluster repeat")
 
 
 def test_bf16_C2_full():
