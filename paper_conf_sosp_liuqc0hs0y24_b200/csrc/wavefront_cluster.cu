@@ -7,11 +7,12 @@
 // edge) (Table 4 dependence vectors, L307–L317).  With T ≫ D the time edge dominates.  Here one
 // layer's hidden units are split over a thread-block cluster (H/32 CTAs, 32 units each) whose
 // CTAs keep their weight slab resident in shared memory (the reuse of L345–L349, as in
-// wavefront_resident.cu) and hand h_{d,t} to each other through DSMEM: every CTA stages its
-// 32-unit slice of h_{d,t} in shared memory and bulk-copies it (cp.async.bulk shared::cluster,
-// complete_tx on the receiver's mbarrier) into every cluster CTA's recurrent operand buffer.  The
-// receiver's MMA warp waits on that mbarrier — no global-memory round trip, no readiness counter
-// on the time edge.  Depth edges (layer d-1 → d, another cluster) still go through the blocked
+// wavefront_resident.cu) and hand h_{d,t} to each other through DSMEM: every epilogue thread
+// writes its row of the CTA's 32-unit slice of h_{d,t} straight from registers into every cluster
+// CTA's recurrent operand buffer (st.async shared::cluster, each store carrying complete_tx to the
+// receiver's mbarrier).  The receiver's MMA warp waits on that mbarrier — no global-memory round
+// trip, no readiness counter, no staging or CTA barrier on the time edge.  (A first version
+// staged the slice and bulk-copied it, cp.async.bulk shared::cluster: 0.77 us more per step.)  Depth edges (layer d-1 → d, another cluster) still go through the blocked
 // SSA buffer hb + a release/acquire counter, as in the other kernels.
 //
 // Shapes: batch B <= 64 (the tile is M = 128 with rows >= B never stored), H in {128, 256}
@@ -39,7 +40,7 @@ namespace ft {
 #ifdef FT_TRACE
 // development-only (libft_trace.so): per-step %globaltimer stamps of CTA `g_cev_cta`:
 // 0 MMA warp saw hfull, 1 MMA warp committed, 2 epilogue saw tfull, 3 math done, 4 copies issued,
-// 5 x-half ready (MMA warp saw the first xfull of the step)
+// 5 x-half ready (MMA warp saw the first xfull of the step); 4 = the sends were issued
 __device__ unsigned long long g_cev[4096 * 8];
 __device__ int g_cev_cta = 0;
 #define FT_CEV(t, k) do { if (blockIdx.x == g_cev_cta && (t) < 4096) g_cev[(t) * 8 + (k)] = globaltimer_ns(); } while (0)
@@ -76,7 +77,7 @@ struct KMaps {
 };
 
 struct KLayout {  // byte offsets into the 1024-aligned dynamic shared memory
-    int rec0, rec1, xring, w, stage, bars, bias, total;
+    int rec0, rec1, xring, w, bars, bias, total;
 };
 
 __host__ __device__ constexpr KLayout klayout(int H) {
@@ -86,8 +87,7 @@ __host__ __device__ constexpr KLayout klayout(int H) {
     L.rec1 = rec;
     L.xring = 2 * rec;
     L.w = L.xring + XSTAGES * X_BYTES;
-    L.stage = L.w + 2 * (H / KBK) * WCHUNK;
-    L.bars = L.stage + SLICE_BYTES;
+    L.bars = L.w + 2 * (H / KBK) * WCHUNK;
     L.bias = L.bars + 256;
     L.total = L.bias + 4 * KU * 4;
     return L;
@@ -98,19 +98,12 @@ __device__ __forceinline__ uint32_t kpack(float lo, float hi) {
     return *reinterpret_cast<uint32_t*>(&v);
 }
 
-// Bulk copy of `bytes` from this CTA's shared memory into a cluster peer's shared memory; the
-// peer's mbarrier receives complete_tx(bytes).
-__device__ __forceinline__ void bulk_s2cluster(uint32_t dst_cluster, uint32_t src_cta, uint32_t bytes,
-                                               uint32_t mbar_cluster) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            dst_cluster),
-        "r"(src_cta), "r"(bytes), "r"(mbar_cluster)
-        : "memory");
-}
-__device__ __forceinline__ void bulk_commit_and_wait_read() {
-    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+// 16-byte asynchronous store into a cluster peer's shared memory; complete_tx(16) on its mbarrier.
+__device__ __forceinline__ void st_async_v4(uint32_t dst_cluster, uint4 v, uint32_t mbar_cluster) {
+    asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.v4.b32 [%0], {%1, %2, %3, %4}, [%5];" ::"r"(
+                     dst_cluster),
+                 "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(mbar_cluster)
+                 : "memory");
 }
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -128,7 +121,6 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
     uint8_t* rec[2] = {smem + L.rec0, smem + L.rec1};
     uint8_t* xring = smem + L.xring;
     uint8_t* sW = smem + L.w;
-    uint8_t* stage_buf = smem + L.stage;
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem + L.bars);
     uint64_t* xfull = bars;                       // [XSTAGES]
     uint64_t* xempty = bars + XSTAGES;            // [XSTAGES]
@@ -244,6 +236,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
                 const int p = (t - 1) & 1;
                 mbar_wait_warp(&hfull[p], (uint32_t)((t - 1) >> 1) & 1u);
                 if (lane == 0) FT_CEV(t, 0);
+                fence_proxy_async_smem();  // peers' st.async data → this CTA's tensor-core reads
                 tc_fence_after();
                 if (elect_one()) {
                     // re-arm this buffer for h_{t+1}: its senders first need our h_t, which we
@@ -306,31 +299,24 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
                     creg[u0 + v] = fmaf(fg, creg[u0 + v], ig * gh);
                     zi[v] = og * tanh_approx(creg[u0 + v]);  // h
                 }
+                if (sender) FT_CEV(t, 3);
 #pragma unroll
                 for (int v = 0; v < 8; ++v) hp[u0 / 2 + v] = kpack(zi[2 * v], zi[2 * v + 1]);
             }
-            // (1) the time edge first: stage the slice (k-group-major, row r at r*16 in each
-            //     1 KiB k-group block) and bulk-copy it into every cluster CTA's buffer t & 1
-            if (sender) FT_CEV(t, 3);
+            // (1) the time edge first: every thread st.async's its row of the slice (4 x 16 B)
+            //     straight from registers into every cluster CTA's buffer t & 1, each store
+            //     carrying complete_tx(16) to that CTA's hfull[t & 1] (no staging, no barrier)
             if (t + 1 < P.L0) {
-                if (sender) bulk_commit_and_wait_read();  // the previous step's copies read the stage
-                named_bar_sync(1, 64);
+                const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES + (uint32_t)row * 16u;
+                const uint32_t bar_local = smem_u32(&hfull[t & 1]);
+                for (int r = 0; r < CS; ++r) {
+                    const uint32_t dst = mapa_shared(dst_local, (uint32_t)r);
+                    const uint32_t mb = mapa_shared(bar_local, (uint32_t)r);
 #pragma unroll
-                for (int g = 0; g < KU / 8; ++g)
-                    *reinterpret_cast<uint4*>(stage_buf + g * 1024 + row * 16) =
-                        make_uint4(hp[4 * g], hp[4 * g + 1], hp[4 * g + 2], hp[4 * g + 3]);
-                fence_proxy_async_smem();  // generic-proxy writes → the bulk copy's async-proxy reads
-                named_bar_sync(1, 64);
-                if (sender) {
-                    const uint32_t src = smem_u32(stage_buf);
-                    const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES;
-                    const uint32_t bar_local = smem_u32(&hfull[t & 1]);
-                    for (int r = 0; r < CS; ++r)
-                        bulk_s2cluster(mapa_shared(dst_local, (uint32_t)r), src, SLICE_BYTES,
-                                       mapa_shared(bar_local, (uint32_t)r));
-                    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-                    FT_CEV(t, 4);
+                    for (int g = 0; g < KU / 8; ++g)
+                        st_async_v4(dst + g * 1024u, make_uint4(hp[4 * g], hp[4 * g + 1], hp[4 * g + 2], hp[4 * g + 3]), mb);
                 }
+                if (sender) FT_CEV(t, 4);
             }
             // (2) the depth edge: h into the blocked SSA buffer, then one cumulative release
             const Cell cell{d + t, d, t, 0};
@@ -378,7 +364,6 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
             acc ^= 1;
             if (acc == 0) acc_phase ^= 1;
         }
-        if (sender) bulk_commit_and_wait_read();
     }
     tc_fence_before();
     __syncthreads();
