@@ -484,6 +484,11 @@ FT_API ft_status ft_grid_rnn_fwd(int batch, int len_x, int len_y, int hidden, in
 
 FT_API long long ft_wavefront_cells(int kind, int depth, int len_a, int len_b, int* out_cells,
                                     long long cap) {
+    return ft_wavefront_cells_banded(kind, depth, len_a, len_b, 0, 1, out_cells, cap);
+}
+
+FT_API long long ft_wavefront_cells_banded(int kind, int depth, int len_a, int len_b, int band,
+                                           int skew, int* out_cells, long long cap) {
     if (kind != ft::KIND_SEQ && kind != ft::KIND_GRID) return -1;
     if (kind == ft::KIND_SEQ) len_b = 1;
     if (depth <= 0 || len_a <= 0 || len_b <= 0 || depth > FT_MAX_DEPTH) return -1;
@@ -498,6 +503,8 @@ FT_API long long ft_wavefront_cells(int kind, int depth, int len_a, int len_b, i
     p.naxes = kind == ft::KIND_SEQ ? 1 : 2;
     p.MB = p.NT = 1;
     p.ncells = (long long)depth * len_a * len_b;
+    p.band = kind == ft::KIND_SEQ ? band : 0;
+    p.skew = kind == ft::KIND_SEQ ? skew : 1;
     ft::Cursor cur = ft::cursor_begin();
     for (long long o = 0; o < p.ncells; ++o) {
         ft::cursor_seek(p, cur, o);

@@ -45,6 +45,9 @@ struct Problem {
                          // 16 no weight loads, 32 fixed load coordinates, 128 EVICT_NORMAL state;
                          // 64 = stress mode: random delays before each counter release
                          // (results stay valid; used by tests to shake out ordering bugs)
+    int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
+                         // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
+                         // (see next_cell); bands run one after the other
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT
     int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)
@@ -68,18 +71,52 @@ FT_HD Cell first_cell() { return Cell{0, 0, 0, 0}; }
 // Successor of `c` in wavefront order: diagonal ascending; within a diagonal depth ascending,
 // then i ascending.  For KIND_SEQ the cells of diagonal k are d ∈ [max(0, k-L+1), min(k, D-1)]
 // with t = k - d — exactly Table 5's bounds (L355–L358) extended to the boundary regions.
+//
+// KIND_SEQ generalisation (band, skew): the layers are cut into bands of `band` consecutive
+// layers [d0, d0 + nb); band after band, each band runs the hyperplane π = t + skew·(d − d0)
+// (a legal schedule for any skew ≥ 1: both dependence vectors e_depth and s·e_time of Table 4
+// get π-distance ≥ 1, and every cell of an earlier band precedes the band).  band = D, skew = 1
+// is the paper's π = d + t.  A band's weights are what one diagonal reads, so a band that fits in
+// L2 turns the per-diagonal weight stream from HBM into L2 hits; skew 2 makes the layer-input
+// half of a cell's K loop ready one diagonal before its recurrent half.  Cell.k numbers the
+// diagonals globally (bands consecutively).
+FT_HD int seq_band(const Problem& p) { return p.band > 0 && p.band < p.D ? p.band : p.D; }
+FT_HD int seq_skew(const Problem& p) { return p.skew > 1 ? p.skew : 1; }
 FT_HD Cell next_cell(const Problem& p, Cell c) {
     if (p.kind == KIND_SEQ) {
-        const int dhi = imin(c.k, p.D - 1);
-        if (c.d < dhi) {
+        const int nbw = seq_band(p), s = seq_skew(p);
+        int d0 = (c.d / nbw) * nbw;
+        int nb = imin(nbw, p.D - d0);
+        int kl = c.i + s * (c.d - d0);  // band-local diagonal
+        // next depth on the same diagonal
+        if (c.d + 1 < d0 + nb && kl - s * (c.d + 1 - d0) >= 0) {
             c.d += 1;
-        } else {
-            c.k += 1;
-            c.d = imax(0, c.k - p.L0 + 1);
+            c.i = kl - s * (c.d - d0);
+            return c;
         }
-        c.i = c.k - c.d;
-        c.j = 0;
-        return c;
+        // next non-empty diagonal (of this band, else of the next band)
+        for (;;) {
+            c.k += 1;
+            kl += 1;
+            if (kl > p.L0 - 1 + s * (nb - 1)) {
+                d0 += nb;
+                if (d0 >= p.D) {  // past the end: never dereferenced by callers
+                    c.d = p.D;
+                    c.i = 0;
+                    return c;
+                }
+                nb = imin(nbw, p.D - d0);
+                kl = 0;
+            }
+            // smallest e = d - d0 with t = kl - s·e <= L0 - 1
+            int e = kl - (p.L0 - 1) > 0 ? (kl - (p.L0 - 1) + s - 1) / s : 0;
+            if (e <= nb - 1 && kl - s * e >= 0) {
+                c.d = d0 + e;
+                c.i = kl - s * e;
+                c.j = 0;
+                return c;
+            }
+        }
     }
     // KIND_GRID: diagonal k = d + i + j.
     const int r = c.k - c.d;

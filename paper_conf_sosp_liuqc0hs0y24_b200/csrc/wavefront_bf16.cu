@@ -807,6 +807,29 @@ bool persisting_limit_at_least(int dev, size_t bytes, cudaStream_t s) {
     return true;
 }
 
+// Layer bands (a5 when the weight set does not fit in L2, e.g. C3's 256 MiB): the stacked nest
+// runs band after band of `band` layers (ft_common.cuh next_cell), so one diagonal reads only the
+// band's weights — 4 x 16 MiB at H = 1024 — and those stay in L2 (EVICT_LAST) for the band's
+// T + band - 1 diagonals instead of streaming from HBM on every diagonal.  The price is a longer
+// dependency chain (D / band · (T + band − 1) diagonals instead of T + D − 1) and fewer cells per
+// diagonal; the band is the largest whose weights fit in a 64 MiB L2 budget (measured: 5-6 layers
+// of 16 MiB no longer stay resident) and it is used only when a band's diagonal still gives at
+// least 3/4 of the CTA groups a tile.  C3 (same box): 7.44 -> 6.57 ms, the SM clock at the power
+// cap 997 -> 1455 MHz (profiles/r2_band_sweep.txt).  FT_BAND overrides (0 = off).
+int choose_band(const Problem& p, int workers) {
+    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM) return 0;
+    if (const char* e = getenv("FT_BAND")) {
+        const int b = atoi(e);
+        return b > 0 && b < p.D ? b : 0;
+    }
+    if (p.resident_layers >= p.D) return 0;  // the whole weight set already stays in L2
+    const double layer_bytes = 8.0 * p.H * p.H * 2.0;  // W + U of one layer, bf16
+    const int band = (int)((64.0 * 1024 * 1024) / layer_bytes);
+    if (band < 1 || band >= p.D) return 0;
+    if (4ll * band * p.NT * p.MB < 3ll * workers) return 0;
+    return band;
+}
+
 template <int CG, int U>
 cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
     using C = KCfg<CG, U>;
@@ -907,8 +930,14 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     // (profiles/r2_ab_l2_persist.jsonl).  ft_set_l2_persist() sizes or disables it.
     Problem q = p;
     q.persist_layers = 0;
+    q.band = choose_band(p, (int)(grid / CG));
+    if (q.band > 0) {
+        q.resident_layers = p.D;  // every band's weights EVICT_LAST: resident while the band runs
+        if (const char* e = getenv("FT_SKEW")) q.skew = atoi(e);
+    }
     cudaLaunchAttribute attr2[2];
-    if (p.resident_layers == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.persist_layers != 0) {
+    if (q.band == 0 && p.resident_layers == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM &&
+        p.persist_layers != 0) {
         int maxp = 0, maxw = 0;
         cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
         cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, dev);

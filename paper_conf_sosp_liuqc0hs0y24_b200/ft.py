@@ -33,7 +33,7 @@ EXPORTS = (
     "ft_b2b_gemm_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
-    "ft_wavefront_cells",
+    "ft_wavefront_cells", "ft_wavefront_cells_banded",
     "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
 )
 
@@ -95,6 +95,8 @@ def lib():
         L.ft_comm_destroy.argtypes = [_c_vp]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
+        L.ft_wavefront_cells_banded.restype = _c_ll
+        L.ft_wavefront_cells_banded.argtypes = [_c_int] * 6 + [_c_vp, _c_ll]
         _lib = L
     return _lib
 
@@ -200,6 +202,16 @@ def ft_wavefront_cells(kind, depth, len_a, len_b=1):
         raise FTError(FT_ERR_INVALID_ARGUMENT, "bad schedule query")
     buf = (ctypes.c_int * (4 * n))()
     lib().ft_wavefront_cells(kind, depth, len_a, len_b, ctypes.cast(buf, _c_vp), n)
+    return [tuple(buf[4 * k:4 * k + 4]) for k in range(n)]
+
+
+def ft_wavefront_cells_banded(kind, depth, len_a, len_b=1, band=0, skew=1):
+    """Cell order of the layer-banded wavefront (kind 0): list of (diagonal, d, i, j) — host only."""
+    n = lib().ft_wavefront_cells_banded(kind, depth, len_a, len_b, band, skew, None, 0)
+    if n < 0:
+        raise FTError(FT_ERR_INVALID_ARGUMENT, "bad schedule query")
+    buf = (ctypes.c_int * (4 * n))()
+    lib().ft_wavefront_cells_banded(kind, depth, len_a, len_b, band, skew, ctypes.cast(buf, _c_vp), n)
     return [tuple(buf[4 * k:4 * k + 4]) for k in range(n)]
 
 

@@ -119,3 +119,73 @@ def test_assignment_keeps_the_critical_path():
     T, D, tau, lat = 30, 6, 1.0, 2.0
     span = _event_makespan(0, D, T, 1, dil, 16, 74, tau, lat)
     assert span <= (T + D - 1) * (tau + lat), span
+
+
+# ------------------------------------------------------------------ layer-banded orders (kind 0)
+def _banded_cells(D, T, band, skew):
+    return ft.ft_wavefront_cells_banded(0, D, T, 1, band, skew)
+
+
+@pytest.mark.parametrize("D,T,band,skew,dil", [
+    (16, 12, 5, 2, None), (16, 12, 6, 1, None), (7, 3, 3, 2, None), (5, 1, 2, 3, None),
+    (4, 9, 4, 2, None), (6, 10, 4, 2, [1, 2, 4, 8, 16, 32]), (3, 2, 1, 5, None),
+])
+def test_banded_order_is_a_legal_schedule(D, T, band, skew, dil):
+    """Every cell exactly once; every producer (Table 4: (d-1, t) and (d, t - s_d)) strictly
+    before its consumer; diagonal numbers non-decreasing; each band's cells contiguous."""
+    cells = _banded_cells(D, T, band, skew)
+    assert sorted((d, i) for _, d, i, _ in cells) == [(d, t) for d in range(D) for t in range(T)]
+    pos = {(d, i): o for o, (_, d, i, _) in enumerate(cells)}
+    dil = dil or [1] * D
+    for (d, t), o in pos.items():
+        if d > 0:
+            assert pos[(d - 1, t)] < o
+        if t >= dil[d]:
+            assert pos[(d, t - dil[d])] < o
+    ks = [k for k, _, _, _ in cells]
+    assert ks == sorted(ks)
+    bw = band if 0 < band < D else D
+    bands = [d // bw for _, d, _, _ in cells]
+    assert bands == sorted(bands)
+    # inside a band, the diagonal of (d, t) is t + skew·(d - d0) (+ the band's offset)
+    for k, d, t, _ in cells:
+        d0 = (d // bw) * bw
+        first_k = min(kk for kk, dd, _, _ in cells if dd // bw == d // bw)
+        assert k - first_k == t + max(skew, 1) * (d - d0)
+
+
+def test_banded_defaults_equal_the_paper_order():
+    for D, T in [(16, 12), (3, 7), (5, 1), (1, 4)]:
+        ref = ft.ft_wavefront_cells(0, D, T)
+        assert _banded_cells(D, T, 0, 1) == ref
+        assert _banded_cells(D, T, D, 1) == ref
+        assert _banded_cells(D, T, D + 3, 0) == ref
+
+
+def _simulate_cells(cells, dil, tpc, nw):
+    ordinal = {(c[1], c[2]): o for o, c in enumerate(cells)}
+    queues = [[] for _ in range(nw)]
+    for g in range(len(cells) * tpc):
+        queues[g % nw].append(g)
+    left, heads, remaining = [tpc] * len(cells), [0] * nw, len(cells) * tpc
+    while remaining:
+        done = []
+        for w in range(nw):
+            if heads[w] < len(queues[w]):
+                g = queues[w][heads[w]]
+                _, d, t, _ = cells[g // tpc]
+                ps = ([(d - 1, t)] if d > 0 else []) + ([(d, t - dil[d])] if t >= dil[d] else [])
+                if all(left[ordinal[p]] == 0 for p in ps):
+                    done.append((w, g))
+        assert done, "deadlock"
+        for w, g in done:
+            heads[w] += 1
+            left[g // tpc] -= 1
+        remaining -= len(done)
+
+
+@pytest.mark.parametrize("D,T,band,skew,tpc,nw", [
+    (16, 10, 5, 2, 16, 74), (16, 10, 6, 1, 32, 74), (8, 6, 3, 2, 4, 5), (6, 9, 4, 3, 8, 148),
+])
+def test_banded_assignment_is_deadlock_free(D, T, band, skew, tpc, nw):
+    _simulate_cells(_banded_cells(D, T, band, skew), [1] * D, tpc, nw)
