@@ -56,6 +56,7 @@ struct Problem {
 
 struct Cell {
     int k, d, i, j;   // diagonal, depth, position (i = t for KIND_SEQ; j = 0)
+    int d0, kl;       // KIND_SEQ: first layer of the cell's band, band-local diagonal
 };
 
 FT_HD int num_diagonals(const Problem& p) {
@@ -66,7 +67,7 @@ FT_HD int imax(int a, int b) { return a > b ? a : b; }
 FT_HD int imin(int a, int b) { return a < b ? a : b; }
 
 // First cell (k = 0): (0, 0, 0, 0).
-FT_HD Cell first_cell() { return Cell{0, 0, 0, 0}; }
+FT_HD Cell first_cell() { return Cell{0, 0, 0, 0, 0, 0}; }
 
 // Successor of `c` in wavefront order: diagonal ascending; within a diagonal depth ascending,
 // then i ascending.  For KIND_SEQ the cells of diagonal k are d ∈ [max(0, k-L+1), min(k, D-1)]
@@ -84,35 +85,36 @@ FT_HD int seq_band(const Problem& p) { return p.band > 0 && p.band < p.D ? p.ban
 FT_HD int seq_skew(const Problem& p) { return p.skew > 1 ? p.skew : 1; }
 FT_HD Cell next_cell(const Problem& p, Cell c) {
     if (p.kind == KIND_SEQ) {
+        // no integer division on this path (every role of the kernels walks it per tile): the
+        // band start d0 and the band-local diagonal kl are carried in the cell
         const int nbw = seq_band(p), s = seq_skew(p);
-        int d0 = (c.d / nbw) * nbw;
-        int nb = imin(nbw, p.D - d0);
-        int kl = c.i + s * (c.d - d0);  // band-local diagonal
+        int nb = imin(nbw, p.D - c.d0);
         // next depth on the same diagonal
-        if (c.d + 1 < d0 + nb && kl - s * (c.d + 1 - d0) >= 0) {
+        if (c.d + 1 < c.d0 + nb && c.kl - s * (c.d + 1 - c.d0) >= 0) {
             c.d += 1;
-            c.i = kl - s * (c.d - d0);
+            c.i = c.kl - s * (c.d - c.d0);
             return c;
         }
         // next non-empty diagonal (of this band, else of the next band)
         for (;;) {
             c.k += 1;
-            kl += 1;
-            if (kl > p.L0 - 1 + s * (nb - 1)) {
-                d0 += nb;
-                if (d0 >= p.D) {  // past the end: never dereferenced by callers
+            c.kl += 1;
+            if (c.kl > p.L0 - 1 + s * (nb - 1)) {
+                c.d0 += nb;
+                if (c.d0 >= p.D) {  // past the end: never dereferenced by callers
                     c.d = p.D;
                     c.i = 0;
                     return c;
                 }
-                nb = imin(nbw, p.D - d0);
-                kl = 0;
+                nb = imin(nbw, p.D - c.d0);
+                c.kl = 0;
             }
             // smallest e = d - d0 with t = kl - s·e <= L0 - 1
-            int e = kl - (p.L0 - 1) > 0 ? (kl - (p.L0 - 1) + s - 1) / s : 0;
-            if (e <= nb - 1 && kl - s * e >= 0) {
-                c.d = d0 + e;
-                c.i = kl - s * e;
+            const int over = c.kl - (p.L0 - 1);
+            const int e = over > 0 ? (s == 1 ? over : (over + s - 1) / s) : 0;
+            if (e <= nb - 1 && c.kl - s * e >= 0) {
+                c.d = c.d0 + e;
+                c.i = c.kl - s * e;
                 c.j = 0;
                 return c;
             }
@@ -154,6 +156,15 @@ FT_HD int tiles_per_cell(const Problem& p) { return p.naxes * p.MB * p.NT; }
 // (cell-granular protocol of the fp32 kernel).
 FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
 
+// Under layer bands the bf16 streaming kernel publishes a cell twice: the h-ready counter
+// flags + cell·MB + m (what the next cells' MMAs read: released as soon as h is stored) and the
+// c-ready counter cflag_index() (the cell state, read only by the c-consumer's epilogue: released
+// after the c stores, off the h → MMA → h chain).  Both complete at flag_target().  Otherwise
+// the h-ready counter covers both.
+FT_HD long long cflag_index(const Problem& p, long long cell, int m) {
+    return (p.ncells + cell) * p.MB + m;
+}
+
 // Tile-granular protocol of the bf16 streaming kernel: one counter per (cell, axis, m-block,
 // N-tile), complete when it reaches flag_mult (the CTAs of the tile).  A consumer's K-chunk kc
 // only needs the producer's units [kc*64, kc*64+64) — one N-tile — so consecutive diagonals
@@ -162,18 +173,23 @@ FT_HD long long tile_flag(const Problem& p, long long cell, int axis, int m, int
     return ((cell * p.naxes + axis) * p.MB + m) * (long long)p.NT + n;
 }
 
-// Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).
+// Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).  Every
+// role of the persistent kernels decodes each of its tiles, so decoding avoids integer division:
+// the cursor carries the first tile of its cell and steps cell by cell.
 struct Cursor {
-    long long ord;  // ordinal of `cell` in wavefront order
+    long long ord;    // ordinal of `cell` in wavefront order
+    long long tile0;  // = ord * tiles_per_cell
     Cell cell;
 };
 
-FT_HD Cursor cursor_begin() { return Cursor{0, first_cell()}; }
+FT_HD Cursor cursor_begin() { return Cursor{0, 0, first_cell()}; }
 
 FT_HD void cursor_seek(const Problem& p, Cursor& cur, long long target_ord) {
+    const int tpc = p.naxes * p.MB * p.NT;
     while (cur.ord < target_ord) {
         cur.cell = next_cell(p, cur.cell);
         ++cur.ord;
+        cur.tile0 += tpc;
     }
 }
 
@@ -185,10 +201,20 @@ struct TileId {
 
 FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
     const int tpc = tiles_per_cell(p);
-    cursor_seek(p, cur, tile / tpc);
-    int w = (int)(tile % tpc);
+    while (tile >= cur.tile0 + tpc) {
+        cur.cell = next_cell(p, cur.cell);
+        ++cur.ord;
+        cur.tile0 += tpc;
+    }
+    int w = (int)(tile - cur.tile0);
     TileId t;
     t.cell = cur.cell;
+    t.axis = 0;
+    t.m = 0;
+    if (p.naxes == 1 && p.MB == 1) {  // the common case: the within-cell index is the N-tile
+        t.n = w;
+        return t;
+    }
     t.n = w % p.NT;
     w /= p.NT;
     t.m = w % p.MB;

@@ -8,6 +8,7 @@
 #include <cstdint>
 
 #include <cuda.h>
+#include <cuda_fp16.h>
 
 #include "ft_common.cuh"
 
@@ -404,6 +405,11 @@ __device__ __forceinline__ float tanh_approx(float x) {
     float y;
     asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
+}
+__device__ __forceinline__ __half2 tanh_approx_h2(__half2 x) {
+    uint32_t r, a = *reinterpret_cast<uint32_t*>(&x);
+    asm("tanh.approx.f16x2 %0, %1;" : "=r"(r) : "r"(a));
+    return *reinterpret_cast<__half2*>(&r);
 }
 __device__ __forceinline__ float sigmoid_approx(float x) {
     return fmaf(0.5f, tanh_approx(0.5f * x), 0.5f);

@@ -463,6 +463,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     // EVICT_FIRST weight stream does not push it out before the next diagonal reads it (ncu, C3:
     // DRAM 30.8 -> 30.1 GB per launch).  FT_DEBUG bit 128 reverts to EVICT_NORMAL (A/B runs).
     const uint64_t pol_state = (P.debug & 128) ? policy_evict_normal() : policy_evict_last();
+    const bool split = P.band > 0;  // h and c published separately (see (2b))
     FT_TR_ROLE;
     for (long long tile = first; tile < P.ntiles; tile += stride) {
         const TileId tl = decode_tile(P, cur, tile);
@@ -479,13 +480,17 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         {
             const int e = threadIdx.x - 64;  // 0 .. 255
             const int slice_b = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
-            if (e < 4 * U) sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + e / U) * P.H + tl.n * U + e % U);
+            // the sigmoid gates' bias is stored halved: σ(z + b) = ½ + ½·tanh(z·½ + b·½), and
+            // fma(z, ½, b·½) rounds exactly like ½·(z + b) (power-of-two scaling commutes with RNE)
+            if (e < 4 * U)
+                sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + e / U) * P.H + tl.n * U + e % U) *
+                           (e < 3 * U ? 0.5f : 1.0f);
         }
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
         //     of the c-producer's counter, published to the other epilogue threads by bar.sync
         FT_TR_BEGIN();
         if (cprod >= 0 && leader_thread && !(P.debug & 1))
-            wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
+            wait_flag_geq(T.flags + (split ? cflag_index(P, cprod, tl.m) : cprod * P.MB + tl.m), target);
         named_bar_sync(1, EPI_THREADS);
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
         float cp[EPI_UNITS];
@@ -559,16 +564,37 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 bg[v] = t3.x; bg[v + 1] = t3.y; bg[v + 2] = t3.z; bg[v + 3] = t3.w;
             }
             float hv[16];
+#ifdef FT_EPI_F16
+            // gate activations two units per MUFU op (tanh.approx.f16x2); c and h stay fp32
+#pragma unroll
+            for (int v = 0; v < 16; v += 2) {
+                const __half2 hh = __floats2half2_rn(0.5f, 0.5f);
+                const float2 ig = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
+                    fmaf(zi[v], 0.5f, bi[v]), fmaf(zi[v + 1], 0.5f, bi[v + 1]))), hh, hh));
+                const float2 fg = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
+                    fmaf(zf[v], 0.5f, bf[v]), fmaf(zf[v + 1], 0.5f, bf[v + 1]))), hh, hh));
+                const float2 og = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
+                    fmaf(zo[v], 0.5f, bo[v]), fmaf(zo[v + 1], 0.5f, bo[v + 1]))), hh, hh));
+                const float2 gh = __half22float2(tanh_approx_h2(__floats2half2_rn(zg[v] + bg[v], zg[v + 1] + bg[v + 1])));
+                const float c0 = fmaf(fg.x, cp[u0 + v], ig.x * gh.x);
+                const float c1 = fmaf(fg.y, cp[u0 + v + 1], ig.y * gh.y);
+                cv[u0 + v] = c0;
+                cv[u0 + v + 1] = c1;
+                hv[v] = og.x * tanh_approx(c0);
+                hv[v + 1] = og.y * tanh_approx(c1);
+            }
+#else
 #pragma unroll
             for (int v = 0; v < 16; ++v) {
-                const float ig = sigmoid_approx(zi[v] + bi[v]);
-                const float fg = sigmoid_approx(zf[v] + bf[v]);
-                const float og = sigmoid_approx(zo[v] + bo[v]);
+                const float ig = fmaf(0.5f, tanh_approx(fmaf(zi[v], 0.5f, bi[v])), 0.5f);
+                const float fg = fmaf(0.5f, tanh_approx(fmaf(zf[v], 0.5f, bf[v])), 0.5f);
+                const float og = fmaf(0.5f, tanh_approx(fmaf(zo[v], 0.5f, bo[v])), 0.5f);
                 const float gh = tanh_approx(zg[v] + bg[v]);
                 const float cn = fmaf(fg, cp[u0 + v], ig * gh);
                 cv[u0 + v] = cn;
                 hv[v] = og * tanh_approx(cn);
             }
+#endif
 #pragma unroll
             for (int w = 0; w < 2; ++w)
                 hp[u0 / 8 + w] = make_uint4(pack_bf16x2(hv[8 * w + 0], hv[8 * w + 1]),
@@ -576,19 +602,22 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                                             pack_bf16x2(hv[8 * w + 4], hv[8 * w + 5]),
                                             pack_bf16x2(hv[8 * w + 6], hv[8 * w + 7]));
             // what downstream cells read — h (blocked SSA buffer hb) and c (ring) — stored per
-            // chunk so the stores overlap the next chunk's math
+            // chunk so the stores overlap the next chunk's math; under layer bands c waits until
+            // h is published (see (2b))
             if (valid) {
                 const int nn = n0 + u0;
                 uint4* hdst = reinterpret_cast<uint4*>(
                     (__nv_bfloat16*)T.hb + hb_row(P, row_h, nn / 64, b) * 64 + (nn % 64));
                 st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
-                float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn);
+                if (!split) {
+                    float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn);
 #pragma unroll
-                for (int v = 0; v < 4; ++v)
-                    st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
-                               make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
-                                          __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
-                               pol_state);
+                    for (int v = 0; v < 4; ++v)
+                        st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
+                                   make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
+                                              __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
+                                   pol_state);
+                }
             }
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_MATH] += clock64() - _e0;
@@ -620,6 +649,24 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #ifdef FT_TRACE
             _acc[TR_E_REL] += clock64() - _e1;
 #endif
+        }
+        // (2b) layer bands (the h → MMA → epilogue chain is the critical path): the cell state
+        //      c' → ring only after h is published, on the c-ready counter (only the
+        //      c-consumer's epilogue waits on it, a whole K loop later).  C3 6.61 -> 6.49 ms
+        //      same-box; without bands (C4) the extra barrier + release cost more (0.95 -> 0.99)
+        if (split && valid) {
+            float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, n0);
+#pragma unroll
+            for (int v = 0; v < EPI_UNITS / 4; ++v)
+                st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
+                           make_uint4(__float_as_uint(cv[4 * v]), __float_as_uint(cv[4 * v + 1]),
+                                      __float_as_uint(cv[4 * v + 2]), __float_as_uint(cv[4 * v + 3])),
+                           pol_state);
+        }
+        if (split) {
+            named_bar_sync(1, EPI_THREADS);
+            if (leader_thread)
+                red_release_gpu_add(T.flags + cflag_index(P, cell_lin(P, c.d, c.i, c.j), tl.m), 1);
         }
         // (3) outputs nobody inside the nest reads
         if (valid) {
