@@ -15,7 +15,8 @@ torch.distributed.gather after each forward; `fused` maps rank 0's output buffer
 
 Prints ONE JSON line on rank 0.  Timing: W untimed warm-ups, then K steps bracketed by
 barrier + cuda synchronize, CUDA events on the launching stream, max over ranks.  L2: the
-inputs (268 MB of weights streamed every diagonal) exceed the 126 MB L2, no flush needed.
+inputs (268 MB of weights) exceed the 126 MB L2, no flush needed: the kernel runs the layers in
+bands of 4 (67 MB of weights), so each step starts by loading band 0's weights from HBM again.
 """
 from __future__ import annotations
 
@@ -45,7 +46,8 @@ def workload_config(n_gpus):
         "depth": c["depth"], "seq_len": c["seq"], "hidden": c["hidden"],
         "per_gpu_batch": c["batch"], "global_batch": c["batch"] * n_gpus,
         "parallelism": f"dp{n_gpus} (batch map sharded, weights replicated)",
-        "l2": "inputs > L2: 268 MB of bf16 weights streamed per diagonal vs 126 MB L2; no flush",
+        "l2": "inputs > L2 (268 MB of bf16 weights vs 126 MB L2), no flush: each step re-reads every "
+              "layer band's weights from HBM (bands of 4 layers stay L2-resident only while they run)",
         "seed": ftgen.config_seed(WORKLOAD),
     }
 

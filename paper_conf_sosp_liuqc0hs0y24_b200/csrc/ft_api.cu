@@ -521,6 +521,41 @@ FT_API long long ft_wavefront_cells_banded(int kind, int depth, int len_a, int l
     return p.ncells;
 }
 
+FT_API long long ft_tile_walk(int depth, int seq, int band, int skew, int owner, int ntiles_n,
+                              int worker, int nworkers, int* out, long long cap) {
+    if (depth <= 0 || seq <= 0 || depth > FT_MAX_DEPTH || ntiles_n <= 0 || nworkers <= 0 ||
+        worker < 0 || worker >= nworkers || (cap > 0 && !out))
+        return -1;
+    ft::Problem p;
+    std::memset(&p, 0, sizeof(p));
+    p.kind = ft::KIND_SEQ;
+    p.D = depth;
+    p.L0 = seq;
+    p.L1 = 1;
+    p.B = p.H = 1;
+    p.naxes = 1;
+    p.MB = 1;
+    p.NT = ntiles_n;
+    p.ncells = (long long)depth * seq;
+    p.ntiles = p.ncells * ntiles_n;
+    p.band = band;
+    p.skew = skew;
+    p.owner = owner && band > 0 && band < depth && ft::seq_band(p) * ntiles_n <= nworkers;
+    for (int d = 0; d < depth; ++d) p.dil[d] = 1;
+    ft::TileWalk w = ft::walk_begin(p, worker, nworkers);
+    ft::TileId tl;
+    long long tid = 0, n = 0;
+    while (ft::walk_next(p, w, tl, tid)) {
+        if (n < cap) {
+            out[3 * n + 0] = tl.cell.d;
+            out[3 * n + 1] = tl.cell.i;
+            out[3 * n + 2] = tl.n;
+        }
+        ++n;
+    }
+    return n;
+}
+
 FT_API ft_status ft_b2b_gemm_fwd(int M, int N, int K, int P, ft_dtype dt, const void* A,
                                  const void* B, const void* C, float* D, void* stream) {
     if (dt != FT_F32 && dt != FT_BF16) return fail(FT_ERR_INVALID_ARGUMENT, "unknown dtype");

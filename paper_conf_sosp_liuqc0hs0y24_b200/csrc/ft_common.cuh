@@ -45,6 +45,9 @@ struct Problem {
                          // 16 no weight loads, 32 fixed load coordinates, 128 EVICT_NORMAL state;
                          // 64 = stress mode: random delays before each counter release
                          // (results stay valid; used by tests to shake out ordering bugs)
+    int l2pol;           // bf16 streaming: L2 eviction-policy overrides, 2 bits each (0 default,
+                         // 1 first, 2 normal, 3 last): weights | state stores << 2 | A loads << 4
+    int owner;           // KIND_SEQ under bands: owner-computes tile assignment (see TileWalk)
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
@@ -220,6 +223,71 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
     t.m = w % p.MB;
     t.axis = w / p.MB;
     return t;
+}
+
+// The tiles one worker (a CTA or a CTA pair) of a persistent kernel processes, in order.
+//  * round-robin (default): tiles w, w + nw, w + 2nw, ... of the global wavefront sequence;
+//  * owner-computes (p.owner, stacked LSTM under layer bands, one m-block): worker w < band·NT
+//    owns the slab (band-local layer e = w / NT, N-tile n = w % NT) and runs it for t = 0 .. T−1
+//    in every band (layer d0 + e).  The pair that reads a weight slab is then the same for the
+//    whole band (one die's L2 caches it) and the cell state of the slab never leaves the
+//    epilogue's registers.  Each worker's sequence follows the dependence order (band, then t),
+//    and every dependence (Table 4) points to an earlier (band, t) of another worker or to the
+//    worker's own previous tile, so co-resident workers cannot deadlock.
+// `tid` identifies the tile for tracing: the global sequence index (round-robin) or
+// cell_lin·NT + n (owner).
+struct TileWalk {
+    Cursor cur;
+    long long tile, stride;
+    int e, n, d0, t;  // owner mode (e < 0: idle worker)
+};
+
+FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
+    TileWalk w;
+    w.cur = cursor_begin();
+    w.tile = worker;
+    w.stride = nworkers;
+    w.e = -1;
+    w.n = 0;
+    w.d0 = 0;
+    w.t = 0;
+    if (p.owner && worker < seq_band(p) * p.NT) {
+        w.e = worker / p.NT;
+        w.n = worker - w.e * p.NT;
+    }
+    return w;
+}
+
+FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) {
+    if (!p.owner) {
+        if (w.tile >= p.ntiles) return false;
+        tl = decode_tile(p, w.cur, w.tile);
+        tid = w.tile;
+        w.tile += w.stride;
+        return true;
+    }
+    if (w.e < 0) return false;
+    const int nbw = seq_band(p);
+    while (w.d0 < p.D && w.e >= imin(nbw, p.D - w.d0)) {  // a short last band without layer e
+        w.d0 += nbw;
+        w.t = 0;
+    }
+    if (w.d0 >= p.D) return false;
+    tl.cell.d = w.d0 + w.e;
+    tl.cell.i = w.t;
+    tl.cell.j = 0;
+    tl.cell.d0 = w.d0;
+    tl.cell.kl = w.t + seq_skew(p) * w.e;
+    tl.cell.k = tl.cell.kl;
+    tl.axis = 0;
+    tl.m = 0;
+    tl.n = w.n;
+    tid = cell_lin(p, tl.cell.d, w.t, 0) * p.NT + w.n;
+    if (++w.t == p.L0) {
+        w.t = 0;
+        w.d0 += nbw;
+    }
+    return true;
 }
 
 // Producer cells of (d, i, j) — the dependence vectors of Table 4 (L307–L317):

@@ -8,7 +8,6 @@
 #include <cstdint>
 
 #include <cuda.h>
-#include <cuda_fp16.h>
 
 #include "ft_common.cuh"
 
@@ -185,6 +184,22 @@ __device__ __forceinline__ void tmem_ld_32x32b_x16(uint32_t taddr, float (&v)[16
         : "memory");
 #pragma unroll
     for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+// 32 lanes x 32 bits, 8 consecutive columns per thread.
+__device__ __forceinline__ void tmem_ld_32x32b_x8(uint32_t taddr, float (&v)[8]) {
+    uint32_t r[8];
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]),
+                   "=r"(r[6]), "=r"(r[7])
+                 : "r"(taddr)
+                 : "memory");
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = __uint_as_float(r[i]);
+}
+template <int N>
+__device__ __forceinline__ void tmem_ld_32x32b(uint32_t taddr, float (&v)[N]) {
+    if constexpr (N == 16) tmem_ld_32x32b_x16(taddr, v);
+    else tmem_ld_32x32b_x8(taddr, v);
 }
 __device__ __forceinline__ void tmem_wait_ld() {
     asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
@@ -405,11 +420,6 @@ __device__ __forceinline__ float tanh_approx(float x) {
     float y;
     asm("tanh.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
-}
-__device__ __forceinline__ __half2 tanh_approx_h2(__half2 x) {
-    uint32_t r, a = *reinterpret_cast<uint32_t*>(&x);
-    asm("tanh.approx.f16x2 %0, %1;" : "=r"(r) : "r"(a));
-    return *reinterpret_cast<__half2*>(&r);
 }
 __device__ __forceinline__ float sigmoid_approx(float x) {
     return fmaf(0.5f, tanh_approx(0.5f * x), 0.5f);

@@ -19,7 +19,8 @@
 //           issues M256 N256 K16 MMAs reading both CTAs' shared memory, so each weight tile is
 //           fetched once per cell for the whole 256-row batch and per-CTA weight traffic halves.
 //
-// Warp roles (352 threads per CTA):
+// Warp roles (352 threads per CTA with the default FT_EPI_WARPS = 8; 16 epilogue warps measured
+// slower: C3 6.30 -> 6.61 ms, C4 0.871 -> 0.903 ms, profiles/r2_ab_epi_warps.txt):
 //   warp 0      weight TMA producer: streams the 64-deep K-chunks of B (no dependencies) into a
 //               STAGES-deep shared-memory ring (mbarriers), running ahead of the wavefront.
 //   warp 10     activation TMA producer: waits the tile's producer cells (readiness counters),
@@ -95,7 +96,16 @@ using namespace sm100;
 constexpr int ROWS = BF16_BM;  // 128 batch rows per CTA = TMEM lanes
 constexpr int BK = 64;         // K per stage = one 128-byte swizzle row of bf16 (A operand)
 constexpr int UK = 16;         // UMMA K for kind::f16
-constexpr int THREADS = 352;  // warp 0 weight TMA, 1 MMA, 2-9 epilogue, 10 activation TMA
+// Epilogue warps: 4 TMEM lane quadrants x EPI_PARTS unit ranges of the tile.
+#ifndef FT_EPI_WARPS
+#define FT_EPI_WARPS 8
+#endif
+constexpr int EPI_WARPS = FT_EPI_WARPS;
+constexpr int EPI_PARTS = EPI_WARPS / 4;
+constexpr int EPI_THREADS = EPI_WARPS * 32;
+constexpr int ACT_WARP = 2 + EPI_WARPS;   // the activation TMA producer
+// warp 0 weight TMA, 1 MMA, 2 .. 1+EPI_WARPS epilogue, ACT_WARP activation TMA
+constexpr int THREADS = 32 * (3 + EPI_WARPS);
 
 // Tile configuration: CG CTAs per tile (1 or a cta_group::2 pair), U hidden units per N-tile
 // (64: N = 256 with 128-byte-swizzled weight atoms; 32: N = 128 with 64-byte swizzle — twice the
@@ -114,7 +124,9 @@ struct KCfg {
     static constexpr int STAGES = (196 * 1024) / STAGE_BYTES;  // 4 / 6 / 6 / 8
     static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024 /* bias */ + 1024 /* align */;
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
-    static constexpr int EPI_UNITS = U / 2;                    // units per epilogue thread
+    static constexpr int EPI_UNITS = U / EPI_PARTS;            // units per epilogue thread
+    // units per TMEM load: 16, or 8 with 16 epilogue warps (register budget of 608 threads)
+    static constexpr int EPI_CH = EPI_UNITS < 16 / EPI_PARTS * 2 ? EPI_UNITS : 16 / EPI_PARTS * 2;
 };
 
 struct Maps {
@@ -123,6 +135,12 @@ struct Maps {
 
 __device__ __forceinline__ int weight_layer(const Problem& P, int slice) {
     return P.kind == KIND_SEQ ? slice : slice >> 1;
+}
+
+// L2 eviction policy from a 2-bit override code (0 = keep `dflt`).
+__device__ __forceinline__ uint64_t l2_policy(int code, uint64_t dflt) {
+    return code == 1 ? policy_evict_first() : code == 2 ? policy_evict_normal()
+                                             : code == 3 ? policy_evict_last() : dflt;
 }
 
 // ------------------------------------------------------------------------------ producer
@@ -191,18 +209,19 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const uint32_t full0 = (CG == 2) ? mapa_shared(smem_u32(full), 0) : smem_u32(full);
     int stage = 0;
     uint32_t phase = 0;
-    Cursor cur = cursor_begin();
     const int target = flag_target(P);
     const int kchunks = P.H / BK;
-    const uint64_t pol_stream = policy_evict_first();
-    const uint64_t pol_keep = policy_evict_last();
-    const uint64_t pol_act = policy_evict_normal();
+    uint64_t pol_stream = policy_evict_first();
+    uint64_t pol_keep = policy_evict_last();
+    const uint64_t pol_act = l2_policy((P.l2pol >> 4) & 3, policy_evict_normal());
+    if (P.l2pol & 3) pol_stream = pol_keep = l2_policy(P.l2pol & 3, pol_keep);
     const bool skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
     const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : CG * C::A_BYTES;
-    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     FT_TR_ROLE;
-    for (long long tile = first; tile < P.ntiles; tile += stride) {
-        const TileId tl = decode_tile(P, cur, tile);
+    TileId tl;
+    long long tile;
+    while (walk_next(P, walk, tl, tile)) {
         Segment seg[3];
         const int ns = segments(P, tl, seg);
         const int nchunks = ns * kchunks;
@@ -270,17 +289,17 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
     uint32_t phase = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
-    Cursor cur = cursor_begin();
     const int kchunks = P.H / BK;
     // A: K-major, SW128: 128-B rows, 8-row groups 1024 B apart (SBO); K step = +32 B.
     // B: MN-major, U-unit swizzle atoms (one per gate) U*64*2 B apart (LBO), 8-k-row groups
     //    8*WROW apart (SBO); K step of 16 rows = 16*WROW.  CG 2: each CTA holds half the atoms.
     const uint64_t adesc0 = make_sdesc(smem_u32(sA), 16, 1024);
     const uint64_t bdesc0 = make_sdesc(smem_u32(sB), U * BK * 2, 8 * C::WROW, C::WLAYOUT);
-    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     FT_TR_ROLE;
-    for (long long tile = first; tile < P.ntiles; tile += stride) {
-        const TileId tl = decode_tile(P, cur, tile);
+    TileId tl;
+    long long tile;
+    while (walk_next(P, walk, tl, tile)) {
         Segment seg[3];
         const int nchunks = segments(P, tl, seg) * kchunks;
         FT_TR_DECL;
@@ -345,10 +364,8 @@ __device__ __forceinline__ uint32_t pack_bf16x2(float lo, float hi) {
     return *reinterpret_cast<uint32_t*>(&v);
 }
 
-// 8 epilogue warps: warp w reads TMEM lane quadrant w % 4 (rows) and unit half (w - 2) / 4
-// (32 of the tile's 64 units); one thread per batch row.
-constexpr int EPI_WARPS = 8;
-constexpr int EPI_THREADS = EPI_WARPS * 32;
+// Epilogue warp w reads TMEM lane quadrant w % 4 (rows) and unit range (w - 2) / 4 (U /
+// EPI_PARTS of the tile's U units); one thread per batch row.
 
 // Listing 1's linear cell: y = z + s, s = the previous step's output (fp32 ring), 0 at t = 0.
 // The 256 accumulator columns are 256 consecutive units; warp half h takes columns h*128 ...
@@ -359,36 +376,37 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
     using C = KCfg<CG, U>;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3, half = (warp - 2) >> 2, row = q * 32 + lane;
+    constexpr int COLS = 4 * C::BNU / EPI_PARTS;  // accumulator columns per warp
     const bool leader_thread = (threadIdx.x == 64);
     int acc = 0;
     uint32_t acc_phase = 0;
-    Cursor cur = cursor_begin();
     const int target = flag_target(P);
     __nv_bfloat16* ys = (__nv_bfloat16*)T.h_all;
-    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
-    for (long long tile = first; tile < P.ntiles; tile += stride) {
-        const TileId tl = decode_tile(P, cur, tile);
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
+    TileId tl;
+    long long tile;
+    while (walk_next(P, walk, tl, tile)) {
         const Cell c = tl.cell;
         int ci = 0, cj = 0;
         const long long cprod = c_producer(P, tl, &ci, &cj);
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
-        const int n0 = tl.n * 4 * C::BNU + half * 2 * C::BNU;
+        const int n0 = tl.n * 4 * C::BNU + half * COLS;
         if (cprod >= 0 && leader_thread)
             wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
         named_bar_sync(1, EPI_THREADS);
         mbar_wait(&tfull[acc], acc_phase);
         tc_fence_after();
         const uint32_t tbase = tmem_base + (uint32_t)(acc * C::BN) + ((uint32_t)(q * 32) << 16) +
-                               (uint32_t)(half * 2 * C::BNU);
+                               (uint32_t)(half * COLS);
         const int row_h = h_row(P, c.d, c.i, c.j, 0);
 #pragma unroll 1
-        for (int u0 = 0; u0 < 2 * C::BNU; u0 += 16) {
+        for (int u0 = 0; u0 < COLS; u0 += 16) {
             __syncwarp();
             float z[16];
             tmem_ld_32x32b_x16(tbase + u0, z);
             tmem_wait_ld();
-            if (u0 + 16 == 2 * C::BNU) {
+            if (u0 + 16 == COLS) {
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) {
@@ -448,25 +466,34 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     }
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3;                 // TMEM lane quadrant this warp may access
-    const int half = (warp - 2) >> 2;       // which 32 units of the tile
+    const int half = (warp - 2) >> 2;       // which unit range of the tile
+    constexpr int CH = C::EPI_CH;
     const int row = q * 32 + lane;
     const bool leader_thread = (threadIdx.x == 64);
     int acc = 0;
     uint32_t acc_phase = 0;
-    Cursor cur = cursor_begin();
     const int target = flag_target(P);
     __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
     __nv_bfloat16* y = (__nv_bfloat16*)T.y;
     __nv_bfloat16* h_n = (__nv_bfloat16*)T.h_n;
-    const long long first = blockIdx.x / CG, stride = gridDim.x / CG;
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     // L2 priority of the nest's live state (the c ring and the blocked h): EVICT_LAST, so the
     // EVICT_FIRST weight stream does not push it out before the next diagonal reads it (ncu, C3:
     // DRAM 30.8 -> 30.1 GB per launch).  FT_DEBUG bit 128 reverts to EVICT_NORMAL (A/B runs).
-    const uint64_t pol_state = (P.debug & 128) ? policy_evict_normal() : policy_evict_last();
-    const bool split = P.band > 0;  // h and c published separately (see (2b))
+    const uint64_t pol_state = l2_policy((P.l2pol >> 2) & 3,
+                                         (P.debug & 128) ? policy_evict_normal() : policy_evict_last());
+    // owner-computes (TileWalk): this thread's rows x units of the slab are the same in every
+    // tile, so the cell state stays in registers (cst) from step t to t + 1 — no c ring, no
+    // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
+    const bool own = P.owner;
+    const bool split = P.band > 0 && !own;
+    float cst[EPI_UNITS];
+#pragma unroll
+    for (int v = 0; v < EPI_UNITS; ++v) cst[v] = 0.f;
     FT_TR_ROLE;
-    for (long long tile = first; tile < P.ntiles; tile += stride) {
-        const TileId tl = decode_tile(P, cur, tile);
+    TileId tl;
+    long long tile;
+    while (walk_next(P, walk, tl, tile)) {
         const Cell c = tl.cell;
         int ci = 0, cj = 0;
         const long long cprod = c_producer(P, tl, &ci, &cj);
@@ -489,12 +516,15 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
         //     of the c-producer's counter, published to the other epilogue threads by bar.sync
         FT_TR_BEGIN();
-        if (cprod >= 0 && leader_thread && !(P.debug & 1))
+        if (cprod >= 0 && leader_thread && !own && !(P.debug & 1))
             wait_flag_geq(T.flags + (split ? cflag_index(P, cprod, tl.m) : cprod * P.MB + tl.m), target);
         named_bar_sync(1, EPI_THREADS);
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
         float cp[EPI_UNITS];
-        if (cprod >= 0 && valid) {
+        if (own) {
+#pragma unroll
+            for (int v = 0; v < EPI_UNITS; ++v) cp[v] = cprod >= 0 ? cst[v] : 0.f;
+        } else if (cprod >= 0 && valid) {
             const float* src = T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n0);
             const long long vstride = 4ll * P.B;  // next 4 units of the same batch row
 #pragma unroll
@@ -523,23 +553,23 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         float cv[EPI_UNITS];
         const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
 #pragma unroll
-        for (int u0 = 0; u0 < EPI_UNITS; u0 += 16) {
+        for (int u0 = 0; u0 < EPI_UNITS; u0 += CH) {
             __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
-            float zi[16], zf[16], zo[16], zg[16];
+            float zi[CH], zf[CH], zo[CH], zg[CH];
             long long _e0 = 0;
 #ifdef FT_TRACE
             _e0 = clock64();
 #endif
-            tmem_ld_32x32b_x16(tbase + 0 * U + u0, zi);
-            tmem_ld_32x32b_x16(tbase + 1 * U + u0, zf);
-            tmem_ld_32x32b_x16(tbase + 2 * U + u0, zo);
-            tmem_ld_32x32b_x16(tbase + 3 * U + u0, zg);
+            tmem_ld_32x32b<CH>(tbase + 0 * U + u0, zi);
+            tmem_ld_32x32b<CH>(tbase + 1 * U + u0, zf);
+            tmem_ld_32x32b<CH>(tbase + 2 * U + u0, zo);
+            tmem_ld_32x32b<CH>(tbase + 3 * U + u0, zg);
             tmem_wait_ld();
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_LDTM] += clock64() - _e0;
             _e0 = clock64();
 #endif
-            if (u0 + 16 == EPI_UNITS) {  // accumulator drained → hand it back to the MMA warp
+            if (u0 + CH == EPI_UNITS) {  // accumulator drained → hand it back to the MMA warp
                 tc_fence_before();
                 __syncwarp();
                 if (lane == 0) {
@@ -551,9 +581,9 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             }
             if (P.debug & 2) continue;
             const int ub = half * EPI_UNITS + u0;  // unit offset inside the tile
-            float bi[16], bf[16], bo[16], bg[16];
+            float bi[CH], bf[CH], bo[CH], bg[CH];
 #pragma unroll
-            for (int v = 0; v < 16; v += 4) {
+            for (int v = 0; v < CH; v += 4) {
                 const float4 t0 = *reinterpret_cast<const float4*>(sbias + 0 * U + ub + v);
                 const float4 t1 = *reinterpret_cast<const float4*>(sbias + 1 * U + ub + v);
                 const float4 t2 = *reinterpret_cast<const float4*>(sbias + 2 * U + ub + v);
@@ -563,29 +593,9 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 bo[v] = t2.x; bo[v + 1] = t2.y; bo[v + 2] = t2.z; bo[v + 3] = t2.w;
                 bg[v] = t3.x; bg[v + 1] = t3.y; bg[v + 2] = t3.z; bg[v + 3] = t3.w;
             }
-            float hv[16];
-#ifdef FT_EPI_F16
-            // gate activations two units per MUFU op (tanh.approx.f16x2); c and h stay fp32
+            float hv[CH];
 #pragma unroll
-            for (int v = 0; v < 16; v += 2) {
-                const __half2 hh = __floats2half2_rn(0.5f, 0.5f);
-                const float2 ig = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
-                    fmaf(zi[v], 0.5f, bi[v]), fmaf(zi[v + 1], 0.5f, bi[v + 1]))), hh, hh));
-                const float2 fg = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
-                    fmaf(zf[v], 0.5f, bf[v]), fmaf(zf[v + 1], 0.5f, bf[v + 1]))), hh, hh));
-                const float2 og = __half22float2(__hfma2(tanh_approx_h2(__floats2half2_rn(
-                    fmaf(zo[v], 0.5f, bo[v]), fmaf(zo[v + 1], 0.5f, bo[v + 1]))), hh, hh));
-                const float2 gh = __half22float2(tanh_approx_h2(__floats2half2_rn(zg[v] + bg[v], zg[v + 1] + bg[v + 1])));
-                const float c0 = fmaf(fg.x, cp[u0 + v], ig.x * gh.x);
-                const float c1 = fmaf(fg.y, cp[u0 + v + 1], ig.y * gh.y);
-                cv[u0 + v] = c0;
-                cv[u0 + v + 1] = c1;
-                hv[v] = og.x * tanh_approx(c0);
-                hv[v + 1] = og.y * tanh_approx(c1);
-            }
-#else
-#pragma unroll
-            for (int v = 0; v < 16; ++v) {
+            for (int v = 0; v < CH; ++v) {
                 const float ig = fmaf(0.5f, tanh_approx(fmaf(zi[v], 0.5f, bi[v])), 0.5f);
                 const float fg = fmaf(0.5f, tanh_approx(fmaf(zf[v], 0.5f, bf[v])), 0.5f);
                 const float og = fmaf(0.5f, tanh_approx(fmaf(zo[v], 0.5f, bo[v])), 0.5f);
@@ -594,9 +604,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 cv[u0 + v] = cn;
                 hv[v] = og * tanh_approx(cn);
             }
-#endif
 #pragma unroll
-            for (int w = 0; w < 2; ++w)
+            for (int w = 0; w < CH / 8; ++w)
                 hp[u0 / 8 + w] = make_uint4(pack_bf16x2(hv[8 * w + 0], hv[8 * w + 1]),
                                             pack_bf16x2(hv[8 * w + 2], hv[8 * w + 3]),
                                             pack_bf16x2(hv[8 * w + 4], hv[8 * w + 5]),
@@ -608,11 +617,14 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 const int nn = n0 + u0;
                 uint4* hdst = reinterpret_cast<uint4*>(
                     (__nv_bfloat16*)T.hb + hb_row(P, row_h, nn / 64, b) * 64 + (nn % 64));
-                st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
-                if (!split) {
+                if constexpr (CH == 16)
+                    st_v8_hint(hdst, hp[u0 / 8], hp[u0 / 8 + 1], pol_state);  // one full sector
+                else
+                    st_v4_hint(hdst, hp[u0 / 8], pol_state);
+                if (!split && !own) {
                     float* cdst = T.c_ring + c_ring_index(P, c.d, c.i, c.j, tl.axis, b, nn);
 #pragma unroll
-                    for (int v = 0; v < 4; ++v)
+                    for (int v = 0; v < CH / 4; ++v)
                         st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
                                    make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
                                               __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
@@ -622,6 +634,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_MATH] += clock64() - _e0;
 #endif
+        }
+        if (own) {
+#pragma unroll
+            for (int v = 0; v < EPI_UNITS; ++v) cst[v] = cv[v];
         }
 #ifdef FT_TRACE
         long long _e1 = clock64();
@@ -733,7 +749,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull[a], 1);
-            mbar_init(&tempty[a], 8 * CG);
+            mbar_init(&tempty[a], EPI_WARPS * CG);
         }
         fence_mbarrier_init();
         tma_prefetch_desc(&M.x);
@@ -753,7 +769,7 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
         if (lane == 0) run_producer<CG, U, true>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
         if (rank == 0) run_mma<CG, U>(P, tmem_base, sA, sB, full, empty, tfull, tempty);  // whole warp
-    } else if (warp == 10) {
+    } else if (warp == ACT_WARP) {
         if (lane == 0) run_producer<CG, U, false>(P, T, M, sA, sB, full, empty, rank);
     } else {
         run_epilogue<CG, U>(P, T, tmem_base, tfull, tempty, rank, sbias);
@@ -978,8 +994,13 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     Problem q = p;
     q.persist_layers = 0;
     q.band = choose_band(p, (int)(grid / CG));
+    if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // experiments
     if (q.band > 0) {
         q.resident_layers = p.D;  // every band's weights EVICT_LAST: resident while the band runs
+        bool unit_dil = true;
+        for (int d = 0; d < p.D; ++d) unit_dil = unit_dil && p.dil[d] == 1;
+        q.owner = unit_dil && p.MB == 1 && p.naxes == 1 && (long long)q.band * p.NT <= grid / CG;
+        if (const char* e = getenv("FT_OWNER")) q.owner = q.owner && atoi(e) != 0;  // A/B
         if (const char* e = getenv("FT_SKEW")) q.skew = atoi(e);
     }
     cudaLaunchAttribute attr2[2];

@@ -33,7 +33,7 @@ EXPORTS = (
     "ft_b2b_gemm_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
-    "ft_wavefront_cells", "ft_wavefront_cells_banded",
+    "ft_wavefront_cells", "ft_wavefront_cells_banded", "ft_tile_walk",
     "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
 )
 
@@ -97,6 +97,8 @@ def lib():
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         L.ft_wavefront_cells_banded.restype = _c_ll
         L.ft_wavefront_cells_banded.argtypes = [_c_int] * 6 + [_c_vp, _c_ll]
+        L.ft_tile_walk.restype = _c_ll
+        L.ft_tile_walk.argtypes = [_c_int] * 8 + [_c_vp, _c_ll]
         _lib = L
     return _lib
 
@@ -213,6 +215,16 @@ def ft_wavefront_cells_banded(kind, depth, len_a, len_b=1, band=0, skew=1):
     buf = (ctypes.c_int * (4 * n))()
     lib().ft_wavefront_cells_banded(kind, depth, len_a, len_b, band, skew, ctypes.cast(buf, _c_vp), n)
     return [tuple(buf[4 * k:4 * k + 4]) for k in range(n)]
+
+
+def ft_tile_walk(depth, seq, band, skew, owner, ntiles_n, worker, nworkers):
+    """One worker's tile sequence [(d, t, n), ...] of the bf16 kernel's walk — host only."""
+    n = lib().ft_tile_walk(depth, seq, band, skew, owner, ntiles_n, worker, nworkers, None, 0)
+    if n < 0:
+        raise FTError(FT_ERR_INVALID_ARGUMENT, "bad tile-walk query")
+    buf = (ctypes.c_int * (3 * max(n, 1)))()
+    lib().ft_tile_walk(depth, seq, band, skew, owner, ntiles_n, worker, nworkers, ctypes.cast(buf, _c_vp), n)
+    return [tuple(buf[3 * k:3 * k + 3]) for k in range(n)]
 
 
 def ft_comm_create(devices):

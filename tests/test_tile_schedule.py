@@ -189,3 +189,55 @@ def _simulate_cells(cells, dil, tpc, nw):
 ])
 def test_banded_assignment_is_deadlock_free(D, T, band, skew, tpc, nw):
     _simulate_cells(_banded_cells(D, T, band, skew), [1] * D, tpc, nw)
+
+
+# ------------------------------------------------------------ the bf16 kernel's per-worker walks
+def _walks(D, T, band, skew, owner, nt, nw):
+    return [ft.ft_tile_walk(D, T, band, skew, owner, nt, w, nw) for w in range(nw)]
+
+
+@pytest.mark.parametrize("D,T,band,skew,nt,nw", [
+    (16, 9, 4, 1, 16, 74), (7, 5, 3, 1, 4, 13), (6, 4, 4, 2, 2, 9), (5, 6, 2, 1, 3, 6),
+])
+def test_owner_walk_covers_every_tile_once_in_dependence_order(D, T, band, skew, nt, nw):
+    """Owner-computes: every (d, t, n) exactly once; a worker keeps one slab (n, layer within
+    the band) and runs t ascending inside a band, bands ascending."""
+    walks = _walks(D, T, band, skew, 1, nt, nw)
+    allt = sorted(x for w in walks for x in w)
+    assert allt == [(d, t, n) for d in range(D) for t in range(T) for n in range(nt)]
+    for w, seq in enumerate(walks):
+        if w >= band * nt:
+            assert seq == []
+            continue
+        assert len({n for _, _, n in seq}) <= 1 and len({d % band for d, _, _ in seq}) <= 1
+        assert seq == sorted(seq, key=lambda x: (x[0] // band, x[1]))
+
+
+@pytest.mark.parametrize("owner", [0, 1])
+def test_walks_are_deadlock_free(owner):
+    """Workers run their walks in order; a tile may complete when its producer cells (d-1, t)
+    and (d, t-1) are complete (all N-tiles).  Must terminate for both assignments."""
+    D, T, band, nt, nw = 12, 7, 4, 8, 37
+    walks = _walks(D, T, band, 1, owner, nt, nw)
+    left = {(d, t): nt for d in range(D) for t in range(T)}
+    heads = [0] * nw
+    while any(heads[w] < len(walks[w]) for w in range(nw)):
+        done = []
+        for w in range(nw):
+            if heads[w] < len(walks[w]):
+                d, t, n = walks[w][heads[w]]
+                if (d == 0 or left[(d - 1, t)] == 0) and (t == 0 or left[(d, t - 1)] == 0):
+                    done.append(w)
+        assert done, "deadlock"
+        for w in done:
+            d, t, n = walks[w][heads[w]]
+            heads[w] += 1
+            left[(d, t)] -= 1
+
+
+def test_round_robin_walk_matches_the_cell_order():
+    D, T, band, nt, nw = 8, 5, 3, 4, 7
+    cells = ft.ft_wavefront_cells_banded(0, D, T, 1, band, 1)
+    seq = [(c[1], c[2], n) for c in cells for n in range(nt)]
+    for w in range(nw):
+        assert ft.ft_tile_walk(D, T, band, 1, 0, nt, w, nw) == seq[w::nw]

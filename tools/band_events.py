@@ -34,6 +34,9 @@ torch.cuda.synchronize()
 NT = H // units
 cells = ft.ft_wavefront_cells_banded(0, D, T, 1, band, skew)
 ntiles = len(cells) * NT
+owner = os.environ.get("FT_OWNER", "1") != "0" and band > 0
+if owner:  # owner-computes walk: events are indexed by cell_lin * NT + n (d-major, then t)
+    cells = [((d // band) * (T + skew * band) + t + skew * (d % band), d, t, 0) for d in range(D) for t in range(T)]
 EV_K = 8
 buf = (ctypes.c_ulonglong * (ntiles * EV_K))()
 L.ft_debug_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
@@ -46,7 +49,7 @@ for g in range(ntiles):
     k, d, t, _ = cells[g // NT]
     cell_of.append((k, d, t))
     rel[(d, t)] = max(rel.get((d, t), 0.0), ev[g, 4])
-print(f"{name} units={units} band={band} skew={skew}: span {ev[:, 4].max():.1f} us, {ntiles} tiles")
+print(f"{name} units={units} band={band} skew={skew} owner={owner}: span {ev[:, 4].max():.1f} us, {ntiles} tiles")
 bw = band if 0 < band < D else D
 stats = {}
 for g in range(ntiles):
