@@ -265,6 +265,14 @@ __device__ __forceinline__ void cluster_sync() {
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::
                      : "memory");
 }
+// Arrive on a (possibly remote) cluster mbarrier with the default .release.cta semantics.  For
+// hand-offs that only order tcgen05 operations (tcgen05.wait::ld + tcgen05.fence::before_thread_sync
+// before it, e.g. "accumulator drained"): no generic-memory release at cluster scope is needed, and
+// .release.cluster compiles to MEMBAR.ALL.GPU + ERRBAR, which waits for the warp's outstanding
+// global stores (ncu: 19 K of 253 K stall samples of the C3 kernel on that arrive).
+__device__ __forceinline__ void mbar_arrive_remote_cta(uint32_t cluster_addr) {
+    asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
     asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr)
                  : "memory");

@@ -122,7 +122,7 @@ struct KCfg {
     static constexpr int B_BYTES = GATES * U * BK * 2;         // weight atoms of one K chunk
     static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
     static constexpr int STAGES = (196 * 1024) / STAGE_BYTES;  // 4 / 6 / 6 / 8
-    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 1024 /* bias */ + 1024 /* align */;
+    static constexpr int SMEM_BYTES = STAGES * STAGE_BYTES + 256 + 2048 /* bias x 2 */ + 1024 /* align */;
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
     static constexpr int EPI_UNITS = U / EPI_PARTS;            // units per epilogue thread
     // units per TMEM load: 16, or 8 with 16 epilogue warps (register budget of 608 threads)
@@ -413,7 +413,7 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
                     if constexpr (CG == 1)
                         mbar_arrive(&tempty[acc]);
                     else
-                        mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[acc]), 0));
+                        mbar_arrive_remote_cta(mapa_shared(smem_u32(&tempty[acc]), 0));
                 }
             }
             const int n = n0 + u0;
@@ -445,8 +445,8 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
             ydst[1] = hp[1];
         }
         named_bar_sync(1, EPI_THREADS);
-        if (leader_thread)  // one cumulative release after the barrier (as in run_epilogue)
-            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+        if (leader_thread)  // one cumulative release after the barrier: the CTA's EPI_WARPS shares
+            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, EPI_WARPS);
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
@@ -490,6 +490,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     float cst[EPI_UNITS];
 #pragma unroll
     for (int v = 0; v < EPI_UNITS; ++v) cst[v] = 0.f;
+    int tcount = 0;
     FT_TR_ROLE;
     TileId tl;
     long long tile;
@@ -503,14 +504,18 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         FT_TR_DECL;
         // (0) this tile's bias [4 gates][64 units] → shared memory while the MMAs still run (the
         //     L1 is invalidated by every gpu-scope fence, so per-chunk global bias loads would
-        //     go to L2 on the epilogue's critical path)
+        //     go to L2 on the epilogue's critical path).  Two buffers, alternating per tile: a
+        //     warp can only write tile n+2's buffer after the barrier (1) of tile n+1, which
+        //     every warp reaches only after it finished reading tile n's.
+        float* sb = sbias + (tcount & 1) * 256;
+        ++tcount;
         {
             const int e = threadIdx.x - 64;  // 0 .. 255
             const int slice_b = (P.kind == KIND_SEQ) ? c.d : c.d * 2 + tl.axis;
             // the sigmoid gates' bias is stored halved: σ(z + b) = ½ + ½·tanh(z·½ + b·½), and
             // fma(z, ½, b·½) rounds exactly like ½·(z + b) (power-of-two scaling commutes with RNE)
             if (e < 4 * U)
-                sbias[e] = __ldg(T.b + ((long long)slice_b * 4 + e / U) * P.H + tl.n * U + e % U) *
+                sb[e] = __ldg(T.b + ((long long)slice_b * 4 + e / U) * P.H + tl.n * U + e % U) *
                            (e < 3 * U ? 0.5f : 1.0f);
         }
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
@@ -556,9 +561,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         for (int u0 = 0; u0 < EPI_UNITS; u0 += CH) {
             __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
             float zi[CH], zf[CH], zo[CH], zg[CH];
-            long long _e0 = 0;
 #ifdef FT_TRACE
-            _e0 = clock64();
+            long long _e0 = clock64();
 #endif
             tmem_ld_32x32b<CH>(tbase + 0 * U + u0, zi);
             tmem_ld_32x32b<CH>(tbase + 1 * U + u0, zf);
@@ -576,7 +580,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                     if constexpr (CG == 1)
                         mbar_arrive(&tempty[acc]);
                     else
-                        mbar_arrive_cluster(mapa_shared(smem_u32(&tempty[acc]), 0));
+                        mbar_arrive_remote_cta(mapa_shared(smem_u32(&tempty[acc]), 0));
                 }
             }
             if (P.debug & 2) continue;
@@ -584,10 +588,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             float bi[CH], bf[CH], bo[CH], bg[CH];
 #pragma unroll
             for (int v = 0; v < CH; v += 4) {
-                const float4 t0 = *reinterpret_cast<const float4*>(sbias + 0 * U + ub + v);
-                const float4 t1 = *reinterpret_cast<const float4*>(sbias + 1 * U + ub + v);
-                const float4 t2 = *reinterpret_cast<const float4*>(sbias + 2 * U + ub + v);
-                const float4 t3 = *reinterpret_cast<const float4*>(sbias + 3 * U + ub + v);
+                const float4 t0 = *reinterpret_cast<const float4*>(sb + 0 * U + ub + v);
+                const float4 t1 = *reinterpret_cast<const float4*>(sb + 1 * U + ub + v);
+                const float4 t2 = *reinterpret_cast<const float4*>(sb + 2 * U + ub + v);
+                const float4 t3 = *reinterpret_cast<const float4*>(sb + 3 * U + ub + v);
                 bi[v] = t0.x; bi[v + 1] = t0.y; bi[v + 2] = t0.z; bi[v + 3] = t0.w;
                 bf[v] = t1.x; bf[v + 1] = t1.y; bf[v + 2] = t1.z; bf[v + 3] = t1.w;
                 bo[v] = t2.x; bo[v + 1] = t2.y; bo[v + 2] = t2.z; bo[v + 3] = t2.w;
@@ -642,24 +646,28 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #ifdef FT_TRACE
         long long _e1 = clock64();
 #endif
-        // (2) publish: every epilogue thread's h / c stores are ordered before the leader's
-        //     release by bar.sync (the release is cumulative)
+        // (2) publish: each epilogue warp releases its share of the counter as soon as its own
+        //     h (and, without bands, c) stores are done — no CTA barrier, so no warp waits for
+        //     the slowest one and the release fences of the 8 warps overlap (the counter
+        //     completes at CG · EPI_WARPS increments per tile)
         const long long hi = h_all_index(P, c, tl.axis, b, n0);
 #ifdef FT_TRACE
         if (leader_thread) _acc[TR_E_STORE] += clock64() - _e1;
         _e1 = clock64();
 #endif
-        named_bar_sync(1, EPI_THREADS);
+        __syncwarp();  // orders the warp's stores before lane 0's release (bar.warp.sync)
 #ifdef FT_TRACE
         if (leader_thread) _acc[TR_E_BAR] += clock64() - _e1;
         _e1 = clock64();
 #endif
-        if (leader_thread) {
+        if (lane == 0) {
             if (P.debug & 64) {  // stress mode (tests): a pseudo-random delay before publishing
-                const uint32_t h = (uint32_t)(tile * 2654435761u) ^ (uint32_t)blockIdx.x * 40503u;
+                const uint32_t h = (uint32_t)(tile * 2654435761u) ^ (uint32_t)(blockIdx.x * 40503u + warp * 977u);
                 __nanosleep(200 + (h & 4095u));
             }
             red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+        }
+        if (leader_thread) {
             FT_TR_END(TR_E_WORK);
             if (rank == 0) FT_EV(tile, 4);
 #ifdef FT_TRACE
@@ -680,8 +688,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                            pol_state);
         }
         if (split) {
-            named_bar_sync(1, EPI_THREADS);
-            if (leader_thread)
+            __syncwarp();
+            if (lane == 0)
                 red_release_gpu_add(T.flags + cflag_index(P, cell_lin(P, c.d, c.i, c.j), tl.m), 1);
         }
         // (3) outputs nobody inside the nest reads
@@ -993,6 +1001,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     // (profiles/r2_ab_l2_persist.jsonl).  ft_set_l2_persist() sizes or disables it.
     Problem q = p;
     q.persist_layers = 0;
+    q.flag_mult = CG * EPI_WARPS;  // every epilogue warp of every CTA of a tile releases once
     q.band = choose_band(p, (int)(grid / CG));
     if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // experiments
     if (q.band > 0) {

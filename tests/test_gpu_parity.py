@@ -496,3 +496,46 @@ def test_bf16_l2_persist_window_under_graph_capture():
     torch.cuda.synchronize()
     rows = [1, 200]
     _check(out, _oracle_stacked(p, rows=rows), torch.bfloat16, OUT, rows=rows, ctx="persist graph")
+
+
+# ------------------------------------------------------------------------- layer bands (a4/a5)
+@pytest.mark.parametrize("B,T,H,D,band,skew,owner", [
+    (256, 6, 128, 6, 4, 1, "1"),    # owner-computes, short last band (6 = 4 + 2)
+    (130, 5, 256, 5, 2, 1, "1"),    # owner, padded batch rows in the CTA pair
+    (256, 1, 128, 3, 2, 1, "1"),    # T = 1: every cell is a boundary cell
+    (256, 7, 128, 6, 4, 2, "1"),    # owner with skew 2
+    (256, 6, 128, 6, 4, 1, "0"),    # round-robin banded (h / c published separately)
+    (200, 5, 192, 5, 3, 2, "0"),    # round-robin, skew 2, ragged batch
+    (100, 6, 128, 4, 2, 1, "1"),    # one-CTA tiles (M = 128) with owner-computes
+])
+def test_bf16_layer_bands(B, T, H, D, band, skew, owner, monkeypatch):
+    """The layer-banded order (bands of `band` layers, each a wavefront π = t + skew·(d − d0))
+    with the owner-computes walk (c in registers) or round-robin (c ring + c-ready counter):
+    every output against the oracle, and bitwise equal to the paper order (same per-cell
+    arithmetic)."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    p = ftgen.stacked_inputs(B, T, H, D, 1717 + band * 10 + skew, "bf16")
+    monkeypatch.setenv("FT_BAND", "0")
+    ref_gpu = _run_stacked(p, torch.bfloat16, want_all=True)
+    monkeypatch.setenv("FT_BAND", str(band))
+    monkeypatch.setenv("FT_SKEW", str(skew))
+    monkeypatch.setenv("FT_OWNER", owner)
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"band {B,T,H,D,band,skew,owner}")
+    for k in ALL:
+        assert torch.equal(got[k], ref_gpu[k]), f"{k}: banded order not bitwise equal to the paper order"
+
+
+def test_bf16_layer_bands_stress(monkeypatch):
+    """Owner-computes under randomly delayed counter releases (stress mode), repeated: bitwise
+    stable."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    monkeypatch.setenv("FT_BAND", "2")
+    p = ftgen.stacked_inputs(256, 6, 128, 5, 1818, "bf16")
+    first = _run_stacked(p, torch.bfloat16, want_all=True)
+    monkeypatch.setenv("FT_DEBUG", "64")
+    for _ in range(2):
+        again = _run_stacked(p, torch.bfloat16, want_all=True)
+        for k in ALL:
+            assert torch.equal(again[k], first[k]), k
+    _check(first, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="band stress")
