@@ -27,6 +27,12 @@ run_seq(256, 2, 1024, 5, torch.bfloat16, resident="0")  # streaming weights (80 
 os.environ["FT_TILE_UNITS"] = "32"
 run_seq(130, 4, 128, 2, torch.bfloat16, resident="0")  # CTA pair, 32-unit tiles
 os.environ.pop("FT_TILE_UNITS")
+for band, owner, skew in (("2", "1", "1"), ("2", "0", "2"), ("3", "1", "2")):  # layer bands
+    os.environ.update(FT_BAND=band, FT_OWNER=owner, FT_SKEW=skew)
+    run_seq(256, 5, 128, 5, torch.bfloat16, resident="0")
+    run_seq(100, 3, 128, 4, torch.bfloat16, resident="0")
+for k in ("FT_BAND", "FT_OWNER", "FT_SKEW"):
+    os.environ.pop(k)
 p = ftgen.stacked_inputs(130, 4, 128, 2, 1, "bf16")       # NEXT-2 layer-sequential schedule
 a = [torch.from_numpy(p[k]).to(dev, torch.bfloat16) for k in ("x", "W", "U")] + [torch.from_numpy(p["b"]).to(dev)]
 ft.stacked_lstm_layerwise(*a, want_all=True)
