@@ -7,6 +7,9 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <mutex>
+#include <algorithm>
+#include <cuda.h>
 
 #include "../../include/ft.h"
 #include "ft_internal.h"
@@ -275,19 +278,66 @@ FT_API ft_status ft_stacked_lstm_fwd(int batch, int seq, int hidden, int depth, 
 }
 
 namespace {
+constexpr int HOSTIO_YCHUNK = 10;  // time steps of y per device→host copy
+
 struct HostIoPlan {
-    size_t x_off, y_off, hn_off, cn_off, inner_off, total;
+    size_t x_off, y_off, hn_off, cn_off, ysig_off, inner_off, total;
+    int nchunks;
 };
 HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, size_t inner) {
     const size_t es = elem_size(dt);
     HostIoPlan h{};
+    h.nchunks = (seq + HOSTIO_YCHUNK - 1) / HOSTIO_YCHUNK;
     h.x_off = 0;
     h.y_off = round_up((size_t)batch * seq * hidden * es, 256);
     h.hn_off = h.y_off + round_up((size_t)batch * seq * hidden * es, 256);
     h.cn_off = h.hn_off + round_up((size_t)batch * depth * hidden * es, 256);
-    h.inner_off = h.cn_off + round_up((size_t)batch * depth * hidden * 4, 256);
+    h.ysig_off = h.cn_off + round_up((size_t)batch * depth * hidden * 4, 256);
+    h.inner_off = h.ysig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
     h.total = h.inner_off + inner;
     return h;
+}
+
+// Per-device copy stream of the host-IO overlap, created once (it lives as long as the process's
+// CUDA context; concurrent calls may share it — each call's copies only wait on its own kernel's
+// counters).  The two events are created per call and released once enqueued (re-entrancy).
+struct HostIoStreams {
+    cudaStream_t copy = nullptr;
+    cudaEvent_t reset = nullptr, done = nullptr;
+};
+typedef CUresult (*StreamWaitValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+
+bool hostio_streams(HostIoStreams* out, StreamWaitValue32Fn* wait_fn) {
+    static HostIoStreams per_dev[64];
+    static StreamWaitValue32Fn fn = nullptr;
+    static std::mutex mu;
+    std::lock_guard<std::mutex> lock(mu);
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return false;
+    if (!fn) {
+        void* ptr = nullptr;
+        cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
+        if (cudaGetDriverEntryPointByVersion("cuStreamWaitValue32", &ptr, 12000, cudaEnableDefault, &q) !=
+                cudaSuccess || q != cudaDriverEntryPointSuccess || !ptr) {
+            cudaGetLastError();
+            return false;
+        }
+        fn = reinterpret_cast<StreamWaitValue32Fn>(ptr);
+    }
+    HostIoStreams& h = per_dev[dev];
+    if (!h.copy && cudaStreamCreateWithFlags(&h.copy, cudaStreamNonBlocking) != cudaSuccess) {
+        cudaGetLastError();
+        h.copy = nullptr;
+        return false;
+    }
+    *out = h;
+    if (cudaEventCreateWithFlags(&out->reset, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&out->done, cudaEventDisableTiming) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    *wait_fn = fn;
+    return true;
 }
 }  // namespace
 
@@ -339,9 +389,53 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     t.y = ws + hp.y_off;
     t.h_n = ws + hp.hn_off;
     t.c_n = reinterpret_cast<float*>(ws + hp.cn_off);
+    // y leaves the device in time chunks while the nest still runs (the top layer finishes its
+    // steps in order): the kernel counts each chunk's stored-and-fenced y tiles in ysig, a copy
+    // stream waits for each count (cuStreamWaitValue32) and copies that chunk, and `s` waits for
+    // the copy stream at the end — so the call stays stream-ordered on `s`.  Kernels that do
+    // not signal (fp32, SMEM-resident, cluster) leave ysig_per_step at 0: y is copied after.
+    HostIoStreams hs;
+    StreamWaitValue32Fn wait_value = nullptr;
+    int per_step = 0, per_chunk = 0;
+    const bool overlap = dt == FT_BF16 && !getenv("FT_HOSTIO_SERIAL") && hostio_streams(&hs, &wait_value);
+    if (overlap) {
+        t.ysig = reinterpret_cast<int*>(ws + hp.ysig_off);
+        t.ychunk = HOSTIO_YCHUNK;
+        t.ysig_per_step = &per_step;
+        t.ysig_per_chunk = &per_chunk;
+        e = cudaMemsetAsync(t.ysig, 0, (size_t)hp.nchunks * sizeof(int), s);
+        if (e == cudaSuccess) e = cudaEventRecord(hs.reset, s);
+        if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("hostio setup: ") + cudaGetErrorString(e));
+    }
     st = run(p, dt, t, ws + hp.inner_off, inner, stream);
-    if (st != FT_OK) return st;
-    e = cudaMemcpyAsync(y_host, ws + hp.y_off, xb, cudaMemcpyDeviceToHost, s);
+    if (st != FT_OK) {
+        if (overlap) {
+            cudaEventDestroy(hs.reset);
+            cudaEventDestroy(hs.done);
+        }
+        return st;
+    }
+    if (per_step > 0) {
+        e = cudaStreamWaitEvent(hs.copy, hs.reset, 0);
+        const size_t row = (size_t)seq * hidden * es;  // one batch row of y
+        for (int c = 0; c < hp.nchunks && e == cudaSuccess; ++c) {
+            const int t0 = c * HOSTIO_YCHUNK, t1 = std::min(seq, t0 + HOSTIO_YCHUNK);
+            CUresult r = wait_value(hs.copy, (CUdeviceptr)(t.ysig + c),
+                                    (cuuint32_t)((per_chunk ? 1 : t1 - t0) * per_step), CU_STREAM_WAIT_VALUE_GEQ);
+            if (r != CUDA_SUCCESS) return fail(FT_ERR_CUDA, "cuStreamWaitValue32 failed: " + std::to_string((int)r));
+            const size_t off = (size_t)t0 * hidden * es;
+            e = cudaMemcpy2DAsync(static_cast<uint8_t*>(y_host) + off, row, ws + hp.y_off + off, row,
+                                  (size_t)(t1 - t0) * hidden * es, batch, cudaMemcpyDeviceToHost, hs.copy);
+        }
+        if (e == cudaSuccess) e = cudaEventRecord(hs.done, hs.copy);
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(s, hs.done, 0);
+    } else {
+        e = cudaMemcpyAsync(y_host, ws + hp.y_off, xb, cudaMemcpyDeviceToHost, s);
+    }
+    if (overlap) {  // destroying an enqueued event is safe: released when it completes
+        cudaEventDestroy(hs.reset);
+        cudaEventDestroy(hs.done);
+    }
     if (e == cudaSuccess) e = cudaMemcpyAsync(h_n_host, ws + hp.hn_off, hb, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("D2H: ") + cudaGetErrorString(e));

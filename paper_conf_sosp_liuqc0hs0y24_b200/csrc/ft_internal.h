@@ -26,6 +26,15 @@ struct Tensors {
     float* c_all = nullptr;  // optional
     float* c_ring = nullptr; // workspace: fp32 cell-state ring
     int* flags = nullptr;    // workspace: readiness counters [ncells][MB]
+    // host-IO overlap (ft_stacked_lstm_fwd_hostio): the bf16 streaming kernel adds 1 to
+    // ysig[t / ychunk] per epilogue warp once its part of y(·, t, ·) is stored and fenced, so a
+    // copy stream can move finished time chunks of y to the host while the nest still runs.
+    int* ysig = nullptr;
+    int ychunk = 0;
+    int* ysig_per_step = nullptr;  // HOST: set by the launcher to the increments per time step
+                                   // (0 = this launch does not signal; copy y after the kernel)
+    int* ysig_per_chunk = nullptr; // HOST: 1 = owner walk: each warp signals once per chunk (its
+                                   // last step of the chunk), so a chunk completes at per_step
 };
 
 // Tile shapes of the two kernels.

@@ -721,6 +721,17 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                     d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
             }
         }
+        // (4) host-IO overlap: this warp's share of y(·, t, ·) is stored → fence at system scope
+        //     (a copy engine reads it) and count it for the copy stream (ft_api.cu hostio)
+        if (top && T.ysig && (!own || c.i % T.ychunk == T.ychunk - 1 || c.i == P.L0 - 1)) {
+            // (owner walk: the same warps store every step of their slab, so one fence at the
+            //  chunk's last step covers the chunk)
+            __syncwarp();
+            if (lane == 0) {
+                fence_acq_rel_sys();
+                red_relaxed_sys_add(T.ysig + c.i / T.ychunk, 1);
+            }
+        }
         acc ^= 1;
         if (acc == 0) acc_phase ^= 1;
     }
@@ -1041,6 +1052,11 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
             cfg.attrs = attr2;
             cfg.numAttrs = 2;
         }
+    }
+    if (t.ysig_per_step) {  // every epilogue warp of every tile of a top-layer cell signals once
+        *t.ysig_per_step = (t.ysig && q.kind == KIND_SEQ && q.cell == CELL_LSTM)
+                               ? q.naxes * q.MB * q.NT * CG * EPI_WARPS : 0;
+        if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner;
     }
     e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);

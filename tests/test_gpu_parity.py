@@ -539,3 +539,39 @@ def test_bf16_layer_bands_stress(monkeypatch):
         for k in ALL:
             assert torch.equal(again[k], first[k]), k
     _check(first, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="band stress")
+
+
+# ------------------------------------------------------------------------- host-buffer call (e2e)
+@pytest.mark.parametrize("B,T,H,D,env", [
+    (256, 23, 128, 6, {"FT_BAND": "2", "FT_RESIDENT": "0"}),                  # bands, owner walk
+    (256, 23, 128, 6, {"FT_BAND": "2", "FT_RESIDENT": "0", "FT_HOSTIO_SERIAL": "1"}),
+    (130, 12, 128, 3, {"FT_RESIDENT": "0"}),                                   # paper order, pair
+    (100, 10, 128, 3, {"FT_RESIDENT": "0"}),                                   # 1-CTA tiles, T = chunk
+    (64, 9, 256, 8, {}),                                                       # cluster/resident: no signal
+])
+def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
+    """ft_stacked_lstm_fwd_hostio (pinned host in/out; y copied to the host in time chunks while
+    the nest still runs, when the kernel signals them) equals the device-buffer call bitwise, and
+    both match the oracle."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    p = ftgen.stacked_inputs(B, T, H, D, 1919 + T, "bf16")
+    bf = torch.bfloat16
+    x, W, U, b = dev(p["x"], bf), dev(p["W"], bf), dev(p["U"], bf), dev(p["b"], torch.float32)
+    ref = ft.stacked_lstm(x, W, U, b)
+    torch.cuda.synchronize()
+    x_h = x.cpu().pin_memory()
+    y_h = torch.full((B, T, H), float("nan"), dtype=bf).pin_memory()
+    hn_h = torch.full((B, D, H), float("nan"), dtype=bf).pin_memory()
+    cn_h = torch.full((B, D, H), float("nan"), dtype=torch.float32).pin_memory()
+    nb = ft.ft_stacked_lstm_hostio_workspace_size(B, T, H, D, ft.FT_BF16)
+    ws = torch.empty(nb, dtype=torch.uint8, device="cuda")
+    s = torch.cuda.Stream()
+    for _ in range(2):  # twice: the per-chunk counters are reset by every call
+        ft.check(ft.ft_stacked_lstm_fwd_hostio(B, T, H, D, ft.FT_BF16, x_h.data_ptr(), W.data_ptr(),
+                                               U.data_ptr(), b.data_ptr(), y_h.data_ptr(), hn_h.data_ptr(),
+                                               cn_h.data_ptr(), ws.data_ptr(), nb, s.cuda_stream))
+        s.synchronize()
+        assert torch.equal(y_h, ref["y"].cpu()) and torch.equal(hn_h, ref["h_n"].cpu())
+        assert torch.equal(cn_h, ref["c_n"].cpu())
+    _check({"y": y_h, "h_n": hn_h, "c_n": cn_h}, _oracle_stacked(p), bf, OUT, ctx=f"hostio {B,T,H,D}")
