@@ -281,7 +281,7 @@ namespace {
 constexpr int HOSTIO_YCHUNK = 10;  // time steps of y per device→host copy
 
 struct HostIoPlan {
-    size_t x_off, y_off, hn_off, cn_off, ysig_off, inner_off, total;
+    size_t x_off, y_off, hn_off, cn_off, ysig_off, xsig_off, inner_off, total;
     int nchunks;
 };
 HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, size_t inner) {
@@ -293,7 +293,8 @@ HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, s
     h.hn_off = h.y_off + round_up((size_t)batch * seq * hidden * es, 256);
     h.cn_off = h.hn_off + round_up((size_t)batch * depth * hidden * es, 256);
     h.ysig_off = h.cn_off + round_up((size_t)batch * depth * hidden * 4, 256);
-    h.inner_off = h.ysig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
+    h.xsig_off = h.ysig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
+    h.inner_off = h.xsig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
     h.total = h.inner_off + inner;
     return h;
 }
@@ -302,40 +303,51 @@ HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, s
 // CUDA context; concurrent calls may share it — each call's copies only wait on its own kernel's
 // counters).  The two events are created per call and released once enqueued (re-entrancy).
 struct HostIoStreams {
-    cudaStream_t copy = nullptr;
-    cudaEvent_t reset = nullptr, done = nullptr;
+    cudaStream_t copy = nullptr;  // device→host y chunks (waits on the kernel's counters)
+    cudaStream_t h2d = nullptr;   // host→device x chunks (never waits on a kernel: no cycle
+                                  // between concurrent calls sharing the streams)
+    cudaEvent_t reset = nullptr, done = nullptr, xdone = nullptr;
 };
 typedef CUresult (*StreamWaitValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*StreamWriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 
-bool hostio_streams(HostIoStreams* out, StreamWaitValue32Fn* wait_fn) {
+bool hostio_streams(HostIoStreams* out, StreamWaitValue32Fn* wait_fn, StreamWriteValue32Fn* write_fn) {
     static HostIoStreams per_dev[64];
     static StreamWaitValue32Fn fn = nullptr;
+    static StreamWriteValue32Fn wfn = nullptr;
     static std::mutex mu;
     std::lock_guard<std::mutex> lock(mu);
     int dev = 0;
     if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return false;
-    if (!fn) {
+    if (!fn || !wfn) {
         void* ptr = nullptr;
-        cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
+        void* wptr = nullptr;
+        cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound, wq = q;
         if (cudaGetDriverEntryPointByVersion("cuStreamWaitValue32", &ptr, 12000, cudaEnableDefault, &q) !=
-                cudaSuccess || q != cudaDriverEntryPointSuccess || !ptr) {
+                cudaSuccess || q != cudaDriverEntryPointSuccess || !ptr ||
+            cudaGetDriverEntryPointByVersion("cuStreamWriteValue32", &wptr, 12000, cudaEnableDefault, &wq) !=
+                cudaSuccess || wq != cudaDriverEntryPointSuccess || !wptr) {
             cudaGetLastError();
             return false;
         }
         fn = reinterpret_cast<StreamWaitValue32Fn>(ptr);
+        wfn = reinterpret_cast<StreamWriteValue32Fn>(wptr);
     }
     HostIoStreams& h = per_dev[dev];
-    if (!h.copy && cudaStreamCreateWithFlags(&h.copy, cudaStreamNonBlocking) != cudaSuccess) {
+    if (!h.copy && (cudaStreamCreateWithFlags(&h.copy, cudaStreamNonBlocking) != cudaSuccess ||
+                    cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking) != cudaSuccess)) {
         cudaGetLastError();
-        h.copy = nullptr;
+        h.copy = h.h2d = nullptr;
         return false;
     }
     *out = h;
     if (cudaEventCreateWithFlags(&out->reset, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&out->done, cudaEventDisableTiming) != cudaSuccess) {
+        cudaEventCreateWithFlags(&out->done, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&out->xdone, cudaEventDisableTiming) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
+    *write_fn = wfn;
     *wait_fn = fn;
     return true;
 }
@@ -379,8 +391,7 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     const size_t es = elem_size(dt);
     const size_t xb = (size_t)batch * seq * hidden * es, hb = (size_t)batch * depth * hidden * es;
     const size_t cb = (size_t)batch * depth * hidden * 4;
-    cudaError_t e = cudaMemcpyAsync(ws + hp.x_off, x_host, xb, cudaMemcpyHostToDevice, s);
-    if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("x H2D: ") + cudaGetErrorString(e));
+    cudaError_t e = cudaSuccess;
     ft::Tensors t;
     t.x = ws + hp.x_off;
     t.W = W;
@@ -394,24 +405,53 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     // stream waits for each count (cuStreamWaitValue32) and copies that chunk, and `s` waits for
     // the copy stream at the end — so the call stays stream-ordered on `s`.  Kernels that do
     // not signal (fp32, SMEM-resident, cluster) leave ysig_per_step at 0: y is copied after.
+    // x likewise enters in time chunks on a second copy stream, each followed by a flag write
+    // (cuStreamWriteValue32) that the streaming kernel's activation producer waits for before
+    // the chunk's first layer-0 load; the kernel then reads x [B][T][H] directly (no pack).
     HostIoStreams hs;
     StreamWaitValue32Fn wait_value = nullptr;
+    StreamWriteValue32Fn write_value = nullptr;
     int per_step = 0, per_chunk = 0;
-    const bool overlap = dt == FT_BF16 && !getenv("FT_HOSTIO_SERIAL") && hostio_streams(&hs, &wait_value);
+    const bool overlap = dt == FT_BF16 && !getenv("FT_HOSTIO_SERIAL") &&
+                         ft::bf16_kernel_choice(p) == 2 && hostio_streams(&hs, &wait_value, &write_value);
     if (overlap) {
         t.ysig = reinterpret_cast<int*>(ws + hp.ysig_off);
         t.ychunk = HOSTIO_YCHUNK;
         t.ysig_per_step = &per_step;
         t.ysig_per_chunk = &per_chunk;
-        e = cudaMemsetAsync(t.ysig, 0, (size_t)hp.nchunks * sizeof(int), s);
+        t.xsig = reinterpret_cast<int*>(ws + hp.xsig_off);
+        t.xchunk = HOSTIO_YCHUNK;
+        e = cudaMemsetAsync(t.ysig, 0, (size_t)(hp.xsig_off - hp.ysig_off) + (size_t)hp.nchunks * sizeof(int), s);
         if (e == cudaSuccess) e = cudaEventRecord(hs.reset, s);
-        if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("hostio setup: ") + cudaGetErrorString(e));
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(hs.h2d, hs.reset, 0);
+        const size_t row = (size_t)seq * hidden * es;
+        for (int c = 0; c < hp.nchunks && e == cudaSuccess; ++c) {
+            const int t0 = c * HOSTIO_YCHUNK, t1 = std::min(seq, t0 + HOSTIO_YCHUNK);
+            const size_t off = (size_t)t0 * hidden * es;
+            e = cudaMemcpy2DAsync(ws + hp.x_off + off, row, static_cast<const uint8_t*>(x_host) + off, row,
+                                  (size_t)(t1 - t0) * hidden * es, batch, cudaMemcpyHostToDevice, hs.h2d);
+            if (e == cudaSuccess &&
+                write_value(hs.h2d, (CUdeviceptr)(t.xsig + c), 1, CU_STREAM_WRITE_VALUE_DEFAULT) != CUDA_SUCCESS)
+                e = cudaErrorUnknown;
+        }
+        if (e == cudaSuccess) e = cudaEventRecord(hs.xdone, hs.h2d);
+        if (e != cudaSuccess) {
+            cudaEventDestroy(hs.reset);
+            cudaEventDestroy(hs.done);
+            cudaEventDestroy(hs.xdone);
+            return fail(FT_ERR_CUDA, std::string("hostio setup: ") + cudaGetErrorString(e));
+        }
+    } else {
+        e = cudaMemcpyAsync(ws + hp.x_off, x_host, xb, cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("x H2D: ") + cudaGetErrorString(e));
     }
     st = run(p, dt, t, ws + hp.inner_off, inner, stream);
     if (st != FT_OK) {
-        if (overlap) {
+        if (overlap) {  // x copies are already enqueued; keep `s` ordered after them
+            cudaStreamWaitEvent(s, hs.xdone, 0);
             cudaEventDestroy(hs.reset);
             cudaEventDestroy(hs.done);
+            cudaEventDestroy(hs.xdone);
         }
         return st;
     }
@@ -433,8 +473,10 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
         e = cudaMemcpyAsync(y_host, ws + hp.y_off, xb, cudaMemcpyDeviceToHost, s);
     }
     if (overlap) {  // destroying an enqueued event is safe: released when it completes
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(s, hs.xdone, 0);
         cudaEventDestroy(hs.reset);
         cudaEventDestroy(hs.done);
+        cudaEventDestroy(hs.xdone);
     }
     if (e == cudaSuccess) e = cudaMemcpyAsync(h_n_host, ws + hp.hn_off, hb, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);

@@ -47,6 +47,7 @@ struct Problem {
                          // (results stay valid; used by tests to shake out ordering bugs)
     int l2pol;           // bf16 streaming: L2 eviction-policy overrides, 2 bits each (0 default,
                          // 1 first, 2 normal, 3 last): weights | state stores << 2 | A loads << 4
+    int x_direct;        // bf16 streaming: layer-0 inputs read from x [B][T][H] (host-IO overlap)
     int owner;           // KIND_SEQ under bands: owner-computes tile assignment (see TileWalk)
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
@@ -495,6 +496,22 @@ __device__ __forceinline__ void fence_acq_rel_sys() {
 }
 __device__ __forceinline__ void red_relaxed_sys_add(int* p, int v) {
     asm volatile("red.relaxed.sys.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Bounded acquire-spin (system scope) on a flag written by a copy stream (cuStreamWriteValue32).
+__device__ __forceinline__ int ld_acquire_sys(const int* p) {
+    int v;
+    asm volatile("ld.acquire.sys.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void wait_flag_geq_sys(const int* p, int target) {
+    if (ld_acquire_sys(p) >= target) return;
+    const uint64_t t0 = globaltimer_ns();
+    for (;;) {
+        __nanosleep(256);
+        if (ld_acquire_sys(p) >= target) return;
+        if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
+    }
 }
 
 // Bounded acquire-spin on a readiness counter.

@@ -29,6 +29,11 @@ struct Tensors {
     // host-IO overlap (ft_stacked_lstm_fwd_hostio): the bf16 streaming kernel adds 1 to
     // ysig[t / ychunk] per epilogue warp once its part of y(·, t, ·) is stored and fenced, so a
     // copy stream can move finished time chunks of y to the host while the nest still runs.
+    // host-IO overlap of x: x arrives in time chunks from the host (a copy stream sets
+    // xsig[c] = 1 after chunk c); the streaming kernel then reads layer-0 inputs straight from
+    // x [B][T][H] (3-D TMA, no pack) and waits for xsig[t / xchunk] before a chunk's first use.
+    int* xsig = nullptr;
+    int xchunk = 0;
     int* ysig = nullptr;
     int ychunk = 0;
     int* ysig_per_step = nullptr;  // HOST: set by the launcher to the increments per time step
@@ -49,6 +54,9 @@ cudaError_t launch_wavefront_f32(const Problem& p, const Tensors& t, cudaStream_
                                  std::string* err);
 cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
                                   std::string* err);
+// which bf16 kernel launch_wavefront_bf16 runs for `p`: 0 DSMEM cluster, 1 SMEM-resident,
+// 2 streaming (the only one that honours Tensors::xsig / ysig)
+int bf16_kernel_choice(const Problem& p);
 // NEXT-4 back-to-back GEMMs (b2b_gemm.cu): D[M][64] = (A[M][64] @ B[64][N]) @ C[N][64]
 cudaError_t launch_b2b_gemm(int M, int N, const void* A, const void* B, const void* C, float* D,
                             cudaStream_t s, std::string* err);

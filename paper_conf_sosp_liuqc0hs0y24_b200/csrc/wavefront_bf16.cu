@@ -131,6 +131,7 @@ struct KCfg {
 
 struct Maps {
     CUtensorMap x, ys, h, W, U;
+    CUtensorMap xd;  // x [B][T][H] as (H, T, B), box (64, 1, 128): layer-0 inputs when P.x_direct
 };
 
 __device__ __forceinline__ int weight_layer(const Problem& P, int slice) {
@@ -168,6 +169,10 @@ __device__ __forceinline__ Segment pick(const Segment (&seg)[3], int i) {
 template <int CG>
 __device__ __forceinline__ void load_a(const Problem& P, const Maps& M, uint32_t dst, uint32_t bar,
                                        const Segment& sg, int kc, int arow0, bool fixed, uint64_t pol) {
+    if (sg.src == SRC_X && P.x_direct && !fixed) {  // straight from x [B][T][H] (no pack)
+        tma_load_3d_hint_addr<CG>(dst, &M.xd, bar, kc * BK, sg.row, arow0, pol);
+        return;
+    }
     const CUtensorMap* am = (fixed || sg.src == SRC_X) ? &M.x : (sg.src == SRC_YS ? &M.ys : &M.h);
     tma_load_2d_hint_addr<CG>(dst, am, bar, 0, fixed ? arow0 : (int)hb_row(P, sg.row, kc, arow0), pol);
 }
@@ -246,6 +251,10 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                     wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
                     FT_TR_END(TR_P_FLAG);
                     if (rank == 0) FT_EV(tile, 5);
+                    fence_proxy_async_global();
+                }
+                if (kc == 0 && sg.src == SRC_X && T.xsig) {  // host-IO: this x chunk has landed
+                    wait_flag_geq_sys(T.xsig + sg.row / T.xchunk, 1);
                     fence_proxy_async_global();
                 }
                 if (c == 0 && rank == 0) FT_EV(tile, 1);
@@ -921,6 +930,21 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     const int slices = p.D * p.naxes;
     const int Bp = p.MB * p.BM;
     if (!encode_blocked(enc, &M.x, t.xb, (long long)p.L0 * (p.H / 64) * Bp, err)) return cudaErrorInvalidValue;
+    const bool x_direct = t.xsig != nullptr && p.kind == KIND_SEQ;
+    M.xd = M.x;
+    if (x_direct) {
+        const cuuint64_t dims[3] = {(cuuint64_t)p.H, (cuuint64_t)p.L0, (cuuint64_t)p.B};
+        const cuuint64_t strides[2] = {(cuuint64_t)p.H * 2, (cuuint64_t)p.L0 * p.H * 2};
+        const cuuint32_t box[3] = {(cuuint32_t)BK, 1, (cuuint32_t)ROWS};
+        const cuuint32_t es[3] = {1, 1, 1};
+        CUresult r = enc(&M.xd, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(t.x), dims, strides,
+                         box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) {
+            if (err) *err = "cuTensorMapEncodeTiled(direct x) failed: " + std::to_string((int)r);
+            return cudaErrorInvalidValue;
+        }
+    }
     if (!encode_blocked(enc, &M.ys, p.kind == KIND_GRID ? t.yb : t.xb,
                         (long long)(p.kind == KIND_GRID ? p.L1 : p.L0) * (p.H / 64) * Bp, err))
         return cudaErrorInvalidValue;
@@ -960,7 +984,8 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     {
         const long long nvec = (long long)p.L0 * (p.H / 64) * Bp * 8;
         const int blocks = (int)((nvec + 255) / 256 < 4 * nsm ? (nvec + 255) / 256 : 4 * nsm);
-        pack_rows_kernel<<<blocks, 256, 0, s>>>((const __nv_bfloat16*)t.x, (__nv_bfloat16*)t.xb, p.B, p.L0, p.H, Bp);
+        if (!x_direct)
+            pack_rows_kernel<<<blocks, 256, 0, s>>>((const __nv_bfloat16*)t.x, (__nv_bfloat16*)t.xb, p.B, p.L0, p.H, Bp);
         if (p.kind == KIND_GRID) {
             const long long nv2 = (long long)p.L1 * (p.H / 64) * Bp * 8;
             const int b2 = (int)((nv2 + 255) / 256 < 4 * nsm ? (nv2 + 255) / 256 : 4 * nsm);
@@ -1013,6 +1038,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     Problem q = p;
     q.persist_layers = 0;
     q.flag_mult = CG * EPI_WARPS;  // every epilogue warp of every CTA of a tile releases once
+    q.x_direct = x_direct;
     q.band = choose_band(p, (int)(grid / CG));
     if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // experiments
     if (q.band > 0) {
@@ -1085,22 +1111,31 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned l
 }
 #endif
 
-cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
-                                  std::string* err) {
+int bf16_kernel_choice(const Problem& p) {
     // latency-bound small stacked LSTMs (C2): weights resident in the SMEM of one cluster per
     // layer, h exchanged through DSMEM on the time edge (wavefront_cluster.cu)
     const char* envc = getenv("FT_CLUSTER");  // "0" disables it (comparisons)
     const char* env = getenv("FT_RESIDENT");  // "0" forces the streaming kernel (comparisons)
-    if (!(envc && envc[0] == '0') && !(env && env[0] == '0') && cluster_kernel_applies(p))
-        return launch_wavefront_cluster(p, t, s, err);
+    if (!(envc && envc[0] == '0') && !(env && env[0] == '0') && cluster_kernel_applies(p)) return 0;
     // a5: weights resident in shared memory for the whole sequence when they fit
     if (p.BM == ROWS && !(env && env[0] == '0')) {
         int dev = 0, nsm = 0;
         if (cudaGetDevice(&dev) == cudaSuccess &&
-            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess) {
-            const int bnu = resident_bnu(p, nsm);
-            if (bnu) return launch_wavefront_resident(p, t, s, bnu, err);
-        }
+            cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess &&
+            resident_bnu(p, nsm))
+            return 1;
+    }
+    return 2;
+}
+
+cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream_t s,
+                                  std::string* err) {
+    const int choice = bf16_kernel_choice(p);
+    if (choice == 0) return launch_wavefront_cluster(p, t, s, err);
+    if (choice == 1) {
+        int dev = 0, nsm = 148;
+        if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        return launch_wavefront_resident(p, t, s, resident_bnu(p, nsm), err);
     }
     // N-tile width: 64 units by default; 32 units when a diagonal at 64 units cannot give every
     // CTA group a tile (few cells per diagonal, e.g. the 6-layer dilated C4): twice the tiles, half
