@@ -534,24 +534,27 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             wait_flag_geq(T.flags + (split ? cflag_index(P, cprod, tl.m) : cprod * P.MB + tl.m), target);
         named_bar_sync(1, EPI_THREADS);
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
-        float cp[EPI_UNITS];
+        // cst: the previous c on entry, updated in place to this tile's c' by the math loop
+        // (one register array: the owner walk carries it to the next tile)
         if (own) {
+            if (cprod < 0) {
 #pragma unroll
-            for (int v = 0; v < EPI_UNITS; ++v) cp[v] = cprod >= 0 ? cst[v] : 0.f;
+                for (int v = 0; v < EPI_UNITS; ++v) cst[v] = 0.f;
+            }
         } else if (cprod >= 0 && valid) {
             const float* src = T.c_ring + c_ring_index(P, c.d, ci, cj, tl.axis, b, n0);
             const long long vstride = 4ll * P.B;  // next 4 units of the same batch row
 #pragma unroll
             for (int v = 0; v < EPI_UNITS / 4; ++v) {
                 const float4 t4 = ld_cg_v4_hint(reinterpret_cast<const float4*>(src + v * vstride), pol_state);
-                cp[4 * v + 0] = t4.x;
-                cp[4 * v + 1] = t4.y;
-                cp[4 * v + 2] = t4.z;
-                cp[4 * v + 3] = t4.w;
+                cst[4 * v + 0] = t4.x;
+                cst[4 * v + 1] = t4.y;
+                cst[4 * v + 2] = t4.z;
+                cst[4 * v + 3] = t4.w;
             }
         } else {
 #pragma unroll
-            for (int v = 0; v < EPI_UNITS; ++v) cp[v] = 0.f;
+            for (int v = 0; v < EPI_UNITS; ++v) cst[v] = 0.f;
         }
         FT_TR_BEGIN();
         mbar_wait(&tfull[acc], acc_phase);
@@ -564,7 +567,6 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         const uint32_t tbase = tmem_base + (uint32_t)(acc * C::BN) + ((uint32_t)(q * 32) << 16) +
                                (uint32_t)(half * EPI_UNITS);
         uint4 hp[EPI_UNITS / 8];
-        float cv[EPI_UNITS];
         const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
 #pragma unroll
         for (int u0 = 0; u0 < EPI_UNITS; u0 += CH) {
@@ -613,8 +615,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 const float fg = fmaf(0.5f, tanh_approx(fmaf(zf[v], 0.5f, bf[v])), 0.5f);
                 const float og = fmaf(0.5f, tanh_approx(fmaf(zo[v], 0.5f, bo[v])), 0.5f);
                 const float gh = tanh_approx(zg[v] + bg[v]);
-                const float cn = fmaf(fg, cp[u0 + v], ig * gh);
-                cv[u0 + v] = cn;
+                const float cn = fmaf(fg, cst[u0 + v], ig * gh);
+                cst[u0 + v] = cn;
                 hv[v] = og * tanh_approx(cn);
             }
 #pragma unroll
@@ -639,18 +641,14 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #pragma unroll
                     for (int v = 0; v < CH / 4; ++v)
                         st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
-                                   make_uint4(__float_as_uint(cv[u0 + 4 * v]), __float_as_uint(cv[u0 + 4 * v + 1]),
-                                              __float_as_uint(cv[u0 + 4 * v + 2]), __float_as_uint(cv[u0 + 4 * v + 3])),
+                                   make_uint4(__float_as_uint(cst[u0 + 4 * v]), __float_as_uint(cst[u0 + 4 * v + 1]),
+                                              __float_as_uint(cst[u0 + 4 * v + 2]), __float_as_uint(cst[u0 + 4 * v + 3])),
                                    pol_state);
                 }
             }
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_MATH] += clock64() - _e0;
 #endif
-        }
-        if (own) {
-#pragma unroll
-            for (int v = 0; v < EPI_UNITS; ++v) cst[v] = cv[v];
         }
 #ifdef FT_TRACE
         long long _e1 = clock64();
@@ -692,8 +690,8 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 #pragma unroll
             for (int v = 0; v < EPI_UNITS / 4; ++v)
                 st_v4_hint(reinterpret_cast<uint4*>(cdst + v * 4ll * P.B),
-                           make_uint4(__float_as_uint(cv[4 * v]), __float_as_uint(cv[4 * v + 1]),
-                                      __float_as_uint(cv[4 * v + 2]), __float_as_uint(cv[4 * v + 3])),
+                           make_uint4(__float_as_uint(cst[4 * v]), __float_as_uint(cst[4 * v + 1]),
+                                      __float_as_uint(cst[4 * v + 2]), __float_as_uint(cst[4 * v + 3])),
                            pol_state);
         }
         if (split) {
@@ -712,7 +710,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 float4* d4 = reinterpret_cast<float4*>(T.c_all + hi);
 #pragma unroll
                 for (int v = 0; v < EPI_UNITS / 4; ++v)
-                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+                    d4[v] = make_float4(cst[4 * v], cst[4 * v + 1], cst[4 * v + 2], cst[4 * v + 3]);
             }
             if (top) {
                 uint4* d = reinterpret_cast<uint4*>(y + y_index(P, c, tl.axis, b, n0));
@@ -727,7 +725,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 float4* d4 = reinterpret_cast<float4*>(T.c_n + ni);
 #pragma unroll
                 for (int v = 0; v < EPI_UNITS / 4; ++v)
-                    d4[v] = make_float4(cv[4 * v], cv[4 * v + 1], cv[4 * v + 2], cv[4 * v + 3]);
+                    d4[v] = make_float4(cst[4 * v], cst[4 * v + 1], cst[4 * v + 2], cst[4 * v + 3]);
             }
         }
         // (4) host-IO overlap: this warp's share of y(·, t, ·) is stored → fence at system scope
