@@ -99,7 +99,18 @@ class ClockSampler:
         except Exception:
             self.proc = None
 
-    def stop(self):
+    @staticmethod
+    def _ts(text):
+        # nvidia-smi timestamp "YYYY/MM/DD HH:MM:SS.mmm" (host local time) -> epoch seconds
+        import datetime
+        try:
+            return datetime.datetime.strptime(text.strip(), "%Y/%m/%d %H:%M:%S.%f").timestamp()
+        except ValueError:
+            return None
+
+    def stop(self, window=None):
+        """Stop sampling; summarise the samples taken inside `window` = (t_start, t_end) host
+        epoch seconds (the timed region) when there are any, else the samples under load."""
         if self.proc is None:
             return None
         self.proc.terminate()
@@ -114,7 +125,7 @@ class ClockSampler:
                 if len(parts) < 10:
                     continue
                 try:
-                    rows.append(dict(sm=float(parts[1]), smax=float(parts[2]),
+                    rows.append(dict(ts=self._ts(parts[0]), sm=float(parts[1]), smax=float(parts[2]),
                                      hw=parts[3], hwt=parts[4], swt=parts[5], pc=parts[6],
                                      util=float(parts[7]), pw=float(parts[8]), plim=float(parts[9])))
                 except ValueError:
@@ -122,7 +133,10 @@ class ClockSampler:
         os.unlink(self.path)
         if not rows:
             return None
-        loaded = [r for r in rows if r["util"] > 50] or rows
+        inside = []
+        if window is not None:
+            inside = [r for r in rows if r["ts"] is not None and window[0] - 0.02 <= r["ts"] <= window[1] + 0.02]
+        loaded = inside or [r for r in rows if r["util"] > 50] or rows
         reasons = set()
         for r in loaded:
             for key, name in (("hw", "hw_slowdown"), ("hwt", "hw_thermal_slowdown"),
@@ -135,7 +149,8 @@ class ClockSampler:
                 # sub-second timed region); power.limit is the cap sw_power_cap enforces
                 "power_w_median": statistics.median(r["pw"] for r in loaded),
                 "power_limit_w": max(r["plim"] for r in loaded),
-                "samples": len(loaded)}
+                "samples": len(loaded),
+                "samples_from": "timed region" if inside else "samples under load (none inside the timed region)"}
 
 
 # ----------------------------------------------------------------------------- CPU oracle
@@ -322,6 +337,7 @@ def run_ours(args):
     torch.cuda.synchronize()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)]
+    host_t0 = time.time()
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
     t0.record(stream)
@@ -334,7 +350,9 @@ def run_ours(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    clocks = sampler.stop()
+    host_t1 = time.time()
+    time.sleep(0.06)  # let the sampler write the sample that closes the window
+    clocks = sampler.stop(window=(host_t0, host_t1))
     elapsed_ms = t0.elapsed_time(t1)
     call_ms = [s.elapsed_time(e) for s, e in ev]
     elapsed_ms = max_over_ranks(elapsed_ms)
