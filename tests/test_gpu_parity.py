@@ -336,9 +336,12 @@ def test_bf16_stress_delayed_release(B, T, H, D, dil, monkeypatch):
     _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx="stress")
 
 
-def test_bf16_cuda_graph_capture_replay():
+@pytest.mark.parametrize("band", ["0", "2"])
+def test_bf16_cuda_graph_capture_replay(band, monkeypatch):
     """The forward (counter reset + input pack + persistent kernel) captures into a CUDA graph
-    and replays with new inputs copied into the captured buffers (the serving path)."""
+    and replays with new inputs copied into the captured buffers (the serving path) — in the
+    paper order and in layer bands with the owner-computes walk (C3's schedule)."""
+    monkeypatch.setenv("FT_BAND", band)
     B, T, H, D = 130, 5, 128, 3
     p1 = ftgen.stacked_inputs(B, T, H, D, 1818, "bf16")
     p2 = ftgen.stacked_inputs(B, T, H, D, 1819, "bf16")
@@ -359,7 +362,7 @@ def test_bf16_cuda_graph_capture_replay():
     g.replay()
     torch.cuda.synchronize()
     ref = oracle.stacked_lstm(p2["x"], p1["W"], p1["U"], p1["b"])
-    _check(out, ref, torch.bfloat16, OUT, ctx="graph")
+    _check(out, ref, torch.bfloat16, OUT, ctx=f"graph band={band}")
 
 
 # ------------------------------------------------------------------------- NEXT-4: B2B GEMMs
