@@ -462,7 +462,12 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
             const int t0 = c * HOSTIO_YCHUNK, t1 = std::min(seq, t0 + HOSTIO_YCHUNK);
             CUresult r = wait_value(hs.copy, (CUdeviceptr)(t.ysig + c),
                                     (cuuint32_t)((per_chunk ? 1 : t1 - t0) * per_step), CU_STREAM_WAIT_VALUE_GEQ);
-            if (r != CUDA_SUCCESS) return fail(FT_ERR_CUDA, "cuStreamWaitValue32 failed: " + std::to_string((int)r));
+            if (r != CUDA_SUCCESS) {  // fall back: copy the rest of y on `s` after the kernel
+                e = cudaMemcpy2DAsync(static_cast<uint8_t*>(y_host) + (size_t)t0 * hidden * es, row,
+                                      ws + hp.y_off + (size_t)t0 * hidden * es, row,
+                                      (size_t)(seq - t0) * hidden * es, batch, cudaMemcpyDeviceToHost, s);
+                break;
+            }
             const size_t off = (size_t)t0 * hidden * es;
             e = cudaMemcpy2DAsync(static_cast<uint8_t*>(y_host) + off, row, ws + hp.y_off + off, row,
                                   (size_t)(t1 - t0) * hidden * es, batch, cudaMemcpyDeviceToHost, hs.copy);
