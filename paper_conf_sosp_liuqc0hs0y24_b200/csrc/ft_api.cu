@@ -681,7 +681,9 @@ FT_API long long ft_tile_walk(int depth, int seq, int band, int skew, int owner,
     p.ntiles = p.ncells * ntiles_n;
     p.band = band;
     p.skew = skew;
-    p.owner = owner && band > 0 && band < depth && ft::seq_band(p) * ntiles_n <= nworkers;
+    p.owner = (owner == 1 && band > 0 && band < depth && ft::seq_band(p) * ntiles_n <= nworkers)
+                  ? 1
+                  : (owner == 2 && 2 * ntiles_n <= nworkers ? 2 : 0);
     for (int d = 0; d < depth; ++d) p.dil[d] = 1;
     ft::TileWalk w = ft::walk_begin(p, worker, nworkers);
     ft::TileId tl;

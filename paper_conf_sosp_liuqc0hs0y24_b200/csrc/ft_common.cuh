@@ -48,7 +48,8 @@ struct Problem {
     int l2pol;           // bf16 streaming: L2 eviction-policy overrides, 2 bits each (0 default,
                          // 1 first, 2 normal, 3 last): weights | state stores << 2 | A loads << 4
     int x_direct;        // bf16 streaming: layer-0 inputs read from x [B][T][H] (host-IO overlap)
-    int owner;           // KIND_SEQ under bands: owner-computes tile assignment (see TileWalk)
+    int owner;           // KIND_SEQ tile assignment (see TileWalk): 0 round-robin, 1 owner-computes
+                         // under bands, 2 layer 0 owned (dilated nests) + round-robin for the rest
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
@@ -237,10 +238,19 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
 //    worker's own previous tile, so co-resident workers cannot deadlock.
 // `tid` identifies the tile for tracing: the global sequence index (round-robin) or
 // cell_lin·NT + n (owner).
+//  * layer-0 owners (p.owner == 2, dilated nests whose layer 0 has dilation 1: its T-step
+//    recurrence is the only chain without slack): worker w < NT owns (layer 0, N-tile w) for
+//    t = 0 .. T−1, with its cell state in registers; the other workers take the remaining
+//    tiles round-robin in wavefront order (a subsequence of the paper order, so the argument
+//    above still holds: every dependence points to an earlier tile of the same worker, to a
+//    layer-0 owner, which depends on nothing but its own previous steps, or to an earlier tile
+//    of the global order).
 struct TileWalk {
     Cursor cur;
     long long tile, stride;
-    int e, n, d0, t;  // owner mode (e < 0: idle worker)
+    int e, n, d0, t;     // owner modes (e < 0: idle worker; e == -2: round-robin rest)
+    long long next, idx0;  // p.owner == 2, the rest: next tile index of this worker among the
+                           // non-layer-0 tiles, and that index of the current cell's first tile
 };
 
 FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
@@ -252,9 +262,20 @@ FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
     w.n = 0;
     w.d0 = 0;
     w.t = 0;
-    if (p.owner && worker < seq_band(p) * p.NT) {
+    w.next = 0;
+    w.idx0 = 0;
+    if (p.owner == 1 && worker < seq_band(p) * p.NT) {
         w.e = worker / p.NT;
         w.n = worker - w.e * p.NT;
+    } else if (p.owner == 2) {
+        if (worker < p.NT) {
+            w.e = 0;
+            w.n = worker;
+        } else {
+            w.e = -2;
+            w.next = worker - p.NT;
+            w.stride = nworkers - p.NT;
+        }
     }
     return w;
 }
@@ -265,6 +286,37 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
         tl = decode_tile(p, w.cur, w.tile);
         tid = w.tile;
         w.tile += w.stride;
+        return true;
+    }
+    if (p.owner == 2 && w.e == -2) {  // round-robin over the tiles of layers >= 1
+        const int tpc = tiles_per_cell(p);
+        while (w.cur.ord < p.ncells) {
+            if (w.cur.cell.d != 0) {
+                if (w.next < w.idx0 + tpc) {
+                    tl.cell = w.cur.cell;
+                    tl.axis = 0;
+                    tl.m = 0;
+                    tl.n = (int)(w.next - w.idx0);
+                    tid = w.cur.tile0 + tl.n;
+                    w.next += w.stride;
+                    return true;
+                }
+                w.idx0 += tpc;
+            }
+            w.cur.cell = next_cell(p, w.cur.cell);
+            ++w.cur.ord;
+            w.cur.tile0 += tpc;
+        }
+        return false;
+    }
+    if (p.owner == 2) {  // layer-0 owner
+        if (w.e != 0 || w.t >= p.L0) return false;
+        tl.cell = Cell{w.t, 0, w.t, 0, 0, w.t};
+        tl.axis = 0;
+        tl.m = 0;
+        tl.n = w.n;
+        tid = cell_lin(p, 0, w.t, 0) * p.NT + w.n;
+        ++w.t;
         return true;
     }
     if (w.e < 0) return false;

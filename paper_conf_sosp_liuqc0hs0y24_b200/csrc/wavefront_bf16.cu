@@ -112,7 +112,6 @@ constexpr int THREADS = 32 * (3 + EPI_WARPS);
 // tiles per diagonal at half the per-tile latency, for diagonals too narrow to fill the GPU).
 template <int CG, int U>
 struct KCfg {
-    static constexpr int BNU = U;
     static constexpr int BN = 4 * U;                           // UMMA N (i | f | o | ĝ)
     static constexpr int TMEM_COLS = 2 * BN;                   // double-buffered accumulator
     static constexpr int GATES = 4 / CG;                       // weight gate atoms per CTA
@@ -385,7 +384,7 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
     using C = KCfg<CG, U>;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3, half = (warp - 2) >> 2, row = q * 32 + lane;
-    constexpr int COLS = 4 * C::BNU / EPI_PARTS;  // accumulator columns per warp
+    constexpr int COLS = 4 * U / EPI_PARTS;  // accumulator columns per warp
     const bool leader_thread = (threadIdx.x == 64);
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -400,7 +399,7 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
         const long long cprod = c_producer(P, tl, &ci, &cj);
         const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = b < P.B;
-        const int n0 = tl.n * 4 * C::BNU + half * COLS;
+        const int n0 = tl.n * 4 * U + half * COLS;
         if (cprod >= 0 && leader_thread)
             wait_flag_geq(T.flags + cprod * P.MB + tl.m, target);
         named_bar_sync(1, EPI_THREADS);
@@ -494,7 +493,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     // owner-computes (TileWalk): this thread's rows x units of the slab are the same in every
     // tile, so the cell state stays in registers (cst) from step t to t + 1 — no c ring, no
     // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
-    const bool own = P.owner;
+    const bool own = P.owner == 1 || (P.owner == 2 && (int)(blockIdx.x / CG) < P.NT);
     const bool split = P.band > 0 && !own;
     float cst[EPI_UNITS];
 #pragma unroll
@@ -1038,6 +1037,15 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     q.flag_mult = CG * EPI_WARPS;  // every epilogue warp of every CTA of a tile releases once
     q.x_direct = x_direct;
     q.band = choose_band(p, (int)(grid / CG));
+    // Dedicated owners for layer 0 of a dilated nest (TileWalk owner mode 2: layer 0 has
+    // dilation 1, the only recurrence without slack) measured slower on C4 (0.916-0.920 ->
+    // 0.958 ms, profiles/r2_ab_layer0_owner.txt): the chain is not queueing behind other
+    // layers' tiles.  Opt-in only (FT_OWNER_L0=1).
+    if (const char* e = getenv("FT_OWNER_L0")) {
+        if (atoi(e) != 0 && q.band == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.MB == 1 &&
+            p.naxes == 1 && p.D >= 2 && p.dil[0] == 1 && 2ll * p.NT <= grid / CG)
+            q.owner = 2;
+    }
     if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // experiments
     if (q.band > 0) {
         q.resident_layers = p.D;  // every band's weights EVICT_LAST: resident while the band runs

@@ -578,3 +578,18 @@ def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
         assert torch.equal(y_h, ref["y"].cpu()) and torch.equal(hn_h, ref["h_n"].cpu())
         assert torch.equal(cn_h, ref["c_n"].cpu())
     _check({"y": y_h, "h_n": hn_h, "c_n": cn_h}, _oracle_stacked(p), bf, OUT, ctx=f"hostio {B,T,H,D}")
+
+
+@pytest.mark.parametrize("dil", [[1, 2, 4, 8, 16, 32], [1, 3, 2]])
+def test_bf16_layer0_owner_walk(dil, monkeypatch):
+    """Opt-in layer-0 owners (TileWalk mode 2) for dilated nests: parity and bitwise equality
+    with the default round-robin walk."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    D = len(dil)
+    p = ftgen.stacked_inputs(256, 9, 128, D, 2020 + D, "bf16")
+    ref_gpu = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    monkeypatch.setenv("FT_OWNER_L0", "1")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"l0 owner {dil}")
+    for k in ALL:
+        assert torch.equal(got[k], ref_gpu[k]), k

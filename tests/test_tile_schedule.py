@@ -241,3 +241,37 @@ def test_round_robin_walk_matches_the_cell_order():
     seq = [(c[1], c[2], n) for c in cells for n in range(nt)]
     for w in range(nw):
         assert ft.ft_tile_walk(D, T, band, 1, 0, nt, w, nw) == seq[w::nw]
+
+
+@pytest.mark.parametrize("D,T,nt,nw,dil", [
+    (6, 12, 16, 74, [1, 2, 4, 8, 16, 32]), (3, 7, 4, 11, [1, 3, 2]), (4, 5, 2, 5, [1, 1, 2, 1]),
+])
+def test_layer0_owner_walk(D, T, nt, nw, dil):
+    """Owner mode 2 (dilated nests): workers < nt own layer 0's N-tiles for every t; the rest
+    take the other tiles round-robin in wavefront order.  Coverage, order, deadlock freedom
+    with the dilated dependences (d-1, t) and (d, t - s_d)."""
+    walks = [ft.ft_tile_walk(D, T, 0, 1, 2, nt, w, nw) for w in range(nw)]
+    allt = sorted(x for w in walks for x in w)
+    assert allt == [(d, t, n) for d in range(D) for t in range(T) for n in range(nt)]
+    for w in range(nt):
+        assert walks[w] == [(0, t, w) for t in range(T)]
+    cells = ft.ft_wavefront_cells(0, D, T)
+    order = {(c[1], c[2], n): i for i, c in enumerate(cells) for n in range(nt)}
+    rest = sorted((x for w in walks[nt:] for x in w), key=lambda x: (order[x], x[2]))
+    assert rest == [x for x in sorted(order, key=lambda x: (order[x], x[2])) if x[0] > 0]
+    for w in range(nt, nw):
+        assert walks[w] == rest[w - nt::nw - nt]
+    left = {(d, t): nt for d in range(D) for t in range(T)}
+    heads = [0] * nw
+    while any(heads[w] < len(walks[w]) for w in range(nw)):
+        done = []
+        for w in range(nw):
+            if heads[w] < len(walks[w]):
+                d, t, n = walks[w][heads[w]]
+                if (d == 0 or left[(d - 1, t)] == 0) and (t < dil[d] or left[(d, t - dil[d])] == 0):
+                    done.append(w)
+        assert done, "deadlock"
+        for w in done:
+            d, t, n = walks[w][heads[w]]
+            heads[w] += 1
+            left[(d, t)] -= 1
