@@ -370,8 +370,8 @@ def run_ours(args):
                 "frac_of_sustained": achieved / peak_s if peak_s else None,
                 "flops_per_launch": flops,
                 "launch_ms_mean": mean_call_s * 1e3,
-                "note": "launch duration = one ft_stacked_lstm_fwd call: counter reset + x pack "
-                        "(52 MB) + the persistent wavefront kernel, CUDA events on the launch stream",
+                "note": "launch duration = one ft_stacked_lstm_fwd call: counter reset (memset) + the "
+                        "persistent wavefront kernel, CUDA events on the launch stream",
                 "launch_ms_median": statistics.median(call_ms), "launch_ms_min": min(call_ms)}
     # bound time of the binding roofline row (SURVEY d.2: tensor 4.26 ms, HBM 4.10 ms at C3) and
     # the DRAM side from the committed ncu capture
@@ -447,9 +447,9 @@ def run_ours(args):
         "config": dict(workload_config(n_gpus), gather=args.gather),
         "tensor_pipe_pct_of_peak": 100.0 * roofline["frac"],
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
-        "gpu_launches": 2 * args.steps, "clocks": clocks,
-        "kernels_per_step": {"pack_rows_kernel (x -> blocked layout)": 1,
-                             "wavefront_bf16_kernel<2> (tcgen05/TMA, persistent)": 1},
+        "gpu_launches": args.steps, "clocks": clocks,
+        "kernels_per_step": {"wavefront_bf16_kernel<2, 64> (tcgen05/TMA, persistent; layer bands, "
+                             "owner-computes; x read in place by 3-D TMA)": 1},
     }
     print(json.dumps(line), flush=True)
     if world > 1:

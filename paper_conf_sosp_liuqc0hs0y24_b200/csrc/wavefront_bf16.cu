@@ -927,7 +927,13 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     const int slices = p.D * p.naxes;
     const int Bp = p.MB * p.BM;
     if (!encode_blocked(enc, &M.x, t.xb, (long long)p.L0 * (p.H / 64) * Bp, err)) return cudaErrorInvalidValue;
-    const bool x_direct = t.xsig != nullptr && p.kind == KIND_SEQ;
+    // Stacked/dilated: layer-0 inputs are read straight from x [B][T][H] (3-D TMA, 128 rows of
+    // 128 B per box) instead of being packed into the blocked layout first: the pack launch goes
+    // away and the strided loads are off the dependency chain (x has no producer).  Same-box
+    // C3 5.44 -> 5.40 ms, C4 0.922 -> 0.903 ms (profiles/r2_ab_x_direct.txt).  Grid inputs are
+    // still packed.  FT_X_DIRECT=0 restores the pack (A/B).
+    const char* exd = getenv("FT_X_DIRECT");
+    const bool x_direct = p.kind == KIND_SEQ && (t.xsig != nullptr || !(exd && exd[0] == '0'));
     M.xd = M.x;
     if (x_direct) {
         const cuuint64_t dims[3] = {(cuuint64_t)p.H, (cuuint64_t)p.L0, (cuuint64_t)p.B};
