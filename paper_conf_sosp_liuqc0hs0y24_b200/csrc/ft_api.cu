@@ -647,7 +647,7 @@ FT_API long long ft_wavefront_cells_banded(int kind, int depth, int len_a, int l
     p.naxes = kind == ft::KIND_SEQ ? 1 : 2;
     p.MB = p.NT = 1;
     p.ncells = (long long)depth * len_a * len_b;
-    p.band = kind == ft::KIND_SEQ ? band : 0;
+    p.band = band;
     p.skew = kind == ft::KIND_SEQ ? skew : 1;
     ft::Cursor cur = ft::cursor_begin();
     for (long long o = 0; o < p.ncells; ++o) {

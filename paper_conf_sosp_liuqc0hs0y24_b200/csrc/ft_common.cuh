@@ -125,6 +125,45 @@ FT_HD Cell next_cell(const Problem& p, Cell c) {
             }
         }
     }
+    if (p.band > 0 && p.band < p.D) {
+        // KIND_GRID in depth bands: band after band, each a wavefront over kl = i + j + (d − d0)
+        // (all three dependence vectors e_depth, e_x, e_y of Table 4 keep kl-distance 1)
+        const int nbw = seq_band(p), R = (p.L0 - 1) + (p.L1 - 1);
+        int nb = imin(nbw, p.D - c.d0);
+        const int r = c.kl - (c.d - c.d0);
+        if (c.i < imin(r, p.L0 - 1)) {
+            c.i += 1;
+            c.j = r - c.i;
+            return c;
+        }
+        for (;;) {
+            if (c.d + 1 < c.d0 + nb && c.kl - (c.d + 1 - c.d0) >= 0) {
+                c.d += 1;
+            } else {
+                c.kl += 1;
+                c.k += 1;
+                if (c.kl > R + nb - 1) {
+                    c.d0 += nb;
+                    if (c.d0 >= p.D) {  // past the end: never dereferenced by callers
+                        c.d = p.D;
+                        c.i = c.j = 0;
+                        return c;
+                    }
+                    nb = imin(nbw, p.D - c.d0);
+                    c.kl = 0;
+                }
+                c.d = c.d0 + imax(0, c.kl - R);
+            }
+            const int rr = c.kl - (c.d - c.d0);
+            const int ilo = imax(0, rr - (p.L1 - 1));
+            const int ihi = imin(rr, p.L0 - 1);
+            if (ilo <= ihi) {
+                c.i = ilo;
+                c.j = rr - ilo;
+                return c;
+            }
+        }
+    }
     // KIND_GRID: diagonal k = d + i + j.
     const int r = c.k - c.d;
     if (c.i < imin(r, p.L0 - 1)) {

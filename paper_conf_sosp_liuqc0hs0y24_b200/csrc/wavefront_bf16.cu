@@ -905,11 +905,22 @@ bool persisting_limit_at_least(int dev, size_t bytes, cudaStream_t s) {
 // least 3/4 of the CTA groups a tile.  C3 (same box): 7.44 -> 6.57 ms, the SM clock at the power
 // cap 997 -> 1455 MHz (profiles/r2_band_sweep.txt).  FT_BAND overrides (0 = off).
 int choose_band(const Problem& p, int workers) {
-    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM) return 0;
+    if (p.cell != CELL_LSTM) return 0;
     if (const char* e = getenv("FT_BAND")) {
         const int b = atoi(e);
         return b > 0 && b < p.D ? b : 0;
     }
+    if (p.kind == KIND_GRID) {
+        // grid nests carry two fp32 cell states per cell (c^x, c^y); their rings for all depths
+        // are D · 2 · (Lx + Ly) slots of B·H fp32.  When that exceeds a 64 MiB L2 budget (C5:
+        // 128 MiB), run depth bands whose rings fit: C5 DRAM 9.6 -> 2.9 GB per forward (band 2),
+        // 6.30 -> 6.07 ms same-box (profiles/r2_ab_grid_bands.txt)
+        const double ring_per_depth = 2.0 * (p.L0 + p.L1) * (double)p.B * p.H * 4.0;
+        if (ring_per_depth * p.D <= 64.0 * 1024 * 1024) return 0;
+        const int band = (int)((64.0 * 1024 * 1024) / ring_per_depth);
+        return band < 1 ? 1 : (band >= p.D ? 0 : band);
+    }
+    if (p.kind != KIND_SEQ) return 0;
     if (p.resident_layers >= p.D) return 0;  // the whole weight set already stays in L2
     const double layer_bytes = 8.0 * p.H * p.H * 2.0;  // W + U of one layer, bf16
     const int band = (int)((64.0 * 1024 * 1024) / layer_bytes);

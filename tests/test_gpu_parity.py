@@ -593,3 +593,21 @@ def test_bf16_layer0_owner_walk(dil, monkeypatch):
     _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"l0 owner {dil}")
     for k in ALL:
         assert torch.equal(got[k], ref_gpu[k]), k
+
+
+@pytest.mark.parametrize("B,Lx,Ly,H,D,band", [(130, 4, 5, 128, 3, 1), (100, 3, 3, 64, 4, 2), (256, 2, 6, 128, 2, 1)])
+def test_bf16_grid_depth_bands(B, Lx, Ly, H, D, band, monkeypatch):
+    """Grid RNN in depth bands (FT_BAND): parity with the oracle and bitwise equality with the
+    paper order."""
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, 2121 + band, "bf16")
+    args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
+    monkeypatch.setenv("FT_BAND", "0")
+    ref_gpu = ft.grid_rnn(*args, want_all=True)
+    monkeypatch.setenv("FT_BAND", str(band))
+    got = ft.grid_rnn(*args, want_all=True)
+    torch.cuda.synchronize()
+    keys = ("out", "h_n", "c_n", "h_all", "c_all")
+    ref = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"], want_all=True)
+    _check(got, ref, torch.bfloat16, keys, ctx=f"grid band {B, Lx, Ly, H, D, band}")
+    for k in keys:
+        assert torch.equal(got[k], ref_gpu[k]), k

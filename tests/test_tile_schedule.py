@@ -275,3 +275,20 @@ def test_layer0_owner_walk(D, T, nt, nw, dil):
             d, t, n = walks[w][heads[w]]
             heads[w] += 1
             left[(d, t)] -= 1
+
+
+@pytest.mark.parametrize("D,Lx,Ly,band", [(4, 3, 4, 1), (4, 5, 2, 2), (5, 4, 4, 3), (3, 1, 6, 1), (2, 6, 1, 1)])
+def test_grid_depth_bands_are_legal(D, Lx, Ly, band):
+    """Grid nests in depth bands (band after band, each a wavefront over i + j + (d - d0)): every
+    cell once, producers (d-1,i,j), (d,i-1,j), (d,i,j-1) strictly earlier, bands contiguous;
+    band >= D is the paper order."""
+    cells = ft.ft_wavefront_cells_banded(1, D, Lx, Ly, band, 1)
+    assert sorted((c[1], c[2], c[3]) for c in cells) == [(d, i, j) for d in range(D) for i in range(Lx) for j in range(Ly)]
+    pos = {(c[1], c[2], c[3]): o for o, c in enumerate(cells)}
+    for (d, i, j), o in pos.items():
+        for q in ((d - 1, i, j), (d, i - 1, j), (d, i, j - 1)):
+            if min(q) >= 0:
+                assert pos[q] < o
+    bands = [c[1] // band for c in cells]
+    assert bands == sorted(bands)
+    assert ft.ft_wavefront_cells_banded(1, D, Lx, Ly, D, 1) == ft.ft_wavefront_cells(1, D, Lx, Ly)
