@@ -278,7 +278,14 @@ FT_API ft_status ft_stacked_lstm_fwd(int batch, int seq, int hidden, int depth, 
 }
 
 namespace {
-constexpr int HOSTIO_YCHUNK = 10;  // time steps of y per device→host copy
+// time steps per host-IO chunk (x in, y out): 5 measured best at C3 (exposed copy time per
+// step 0.35 ms vs 0.40 ms at 10 and 0.46 ms at 3, profiles/r2_ab_hostio_chunk.txt);
+// FT_HOSTIO_CHUNK overrides (experiments)
+int hostio_chunk() {
+    const char* e = getenv("FT_HOSTIO_CHUNK");
+    const int c = e ? atoi(e) : 5;
+    return c >= 1 ? c : 5;
+}
 
 struct HostIoPlan {
     size_t x_off, y_off, hn_off, cn_off, ysig_off, xsig_off, inner_off, total;
@@ -287,7 +294,7 @@ struct HostIoPlan {
 HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, size_t inner) {
     const size_t es = elem_size(dt);
     HostIoPlan h{};
-    h.nchunks = (seq + HOSTIO_YCHUNK - 1) / HOSTIO_YCHUNK;
+    h.nchunks = seq;  // room for chunks of 1 step; a call uses ceil(seq / hostio_chunk())
     h.x_off = 0;
     h.y_off = round_up((size_t)batch * seq * hidden * es, 256);
     h.hn_off = h.y_off + round_up((size_t)batch * seq * hidden * es, 256);
@@ -412,21 +419,22 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     StreamWaitValue32Fn wait_value = nullptr;
     StreamWriteValue32Fn write_value = nullptr;
     int per_step = 0, per_chunk = 0;
+    const int chunk = hostio_chunk(), nchunks = (seq + chunk - 1) / chunk;
     const bool overlap = dt == FT_BF16 && !getenv("FT_HOSTIO_SERIAL") &&
                          ft::bf16_kernel_choice(p) == 2 && hostio_streams(&hs, &wait_value, &write_value);
     if (overlap) {
         t.ysig = reinterpret_cast<int*>(ws + hp.ysig_off);
-        t.ychunk = HOSTIO_YCHUNK;
+        t.ychunk = chunk;
         t.ysig_per_step = &per_step;
         t.ysig_per_chunk = &per_chunk;
         t.xsig = reinterpret_cast<int*>(ws + hp.xsig_off);
-        t.xchunk = HOSTIO_YCHUNK;
+        t.xchunk = chunk;
         e = cudaMemsetAsync(t.ysig, 0, (size_t)(hp.xsig_off - hp.ysig_off) + (size_t)hp.nchunks * sizeof(int), s);
         if (e == cudaSuccess) e = cudaEventRecord(hs.reset, s);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(hs.h2d, hs.reset, 0);
         const size_t row = (size_t)seq * hidden * es;
-        for (int c = 0; c < hp.nchunks && e == cudaSuccess; ++c) {
-            const int t0 = c * HOSTIO_YCHUNK, t1 = std::min(seq, t0 + HOSTIO_YCHUNK);
+        for (int c = 0; c < nchunks && e == cudaSuccess; ++c) {
+            const int t0 = c * chunk, t1 = std::min(seq, t0 + chunk);
             const size_t off = (size_t)t0 * hidden * es;
             e = cudaMemcpy2DAsync(ws + hp.x_off + off, row, static_cast<const uint8_t*>(x_host) + off, row,
                                   (size_t)(t1 - t0) * hidden * es, batch, cudaMemcpyHostToDevice, hs.h2d);
@@ -458,8 +466,8 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     if (per_step > 0) {
         e = cudaStreamWaitEvent(hs.copy, hs.reset, 0);
         const size_t row = (size_t)seq * hidden * es;  // one batch row of y
-        for (int c = 0; c < hp.nchunks && e == cudaSuccess; ++c) {
-            const int t0 = c * HOSTIO_YCHUNK, t1 = std::min(seq, t0 + HOSTIO_YCHUNK);
+        for (int c = 0; c < nchunks && e == cudaSuccess; ++c) {
+            const int t0 = c * chunk, t1 = std::min(seq, t0 + chunk);
             CUresult r = wait_value(hs.copy, (CUdeviceptr)(t.ysig + c),
                                     (cuuint32_t)((per_chunk ? 1 : t1 - t0) * per_step), CU_STREAM_WAIT_VALUE_GEQ);
             if (r != CUDA_SUCCESS) {  // fall back: copy the rest of y on `s` after the kernel
