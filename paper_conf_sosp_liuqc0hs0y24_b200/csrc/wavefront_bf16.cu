@@ -1105,7 +1105,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     if (t.ysig_per_step) {  // every epilogue warp of every tile of a top-layer cell signals once
         *t.ysig_per_step = (t.ysig && q.kind == KIND_SEQ && q.cell == CELL_LSTM)
                                ? q.naxes * q.MB * q.NT * CG * EPI_WARPS : 0;
-        if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner;
+        if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner == 1;  // owner walk: once per chunk
     }
     e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);

@@ -551,6 +551,7 @@ def test_bf16_layer_bands_stress(monkeypatch):
     (130, 12, 128, 3, {"FT_RESIDENT": "0"}),                                   # paper order, pair
     (100, 10, 128, 3, {"FT_RESIDENT": "0"}),                                   # 1-CTA tiles, T = chunk
     (64, 9, 256, 8, {}),                                                       # cluster/resident: no signal
+    (256, 12, 128, 4, {"FT_RESIDENT": "0", "FT_OWNER_L0": "1"}),               # layer-0 owners: per-tile y signals
 ])
 def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
     """ft_stacked_lstm_fwd_hostio (pinned host in/out; y copied to the host in time chunks while

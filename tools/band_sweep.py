@@ -13,7 +13,7 @@ sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)) + "/..")
 import ftgen, bench
 from paper_conf_sosp_liuqc0hs0y24_b200 import ft
 
-KEYS = ("FT_BAND", "FT_SKEW", "FT_L2_RESIDENT_LAYERS", "FT_L2_PERSIST_LAYERS", "FT_TILE_UNITS", "FT_L2POL", "FT_DEBUG", "FT_OWNER")
+KEYS = ("FT_BAND", "FT_SKEW", "FT_L2_RESIDENT_LAYERS", "FT_L2_PERSIST_LAYERS", "FT_TILE_UNITS", "FT_L2POL", "FT_DEBUG", "FT_OWNER", "FT_SPLIT_PHASE")
 
 
 def main():
