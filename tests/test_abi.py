@@ -198,3 +198,23 @@ def test_boundary_region_counts():
     assert len(seq) == 4
     grid = {(d > 0, i > 0, j > 0) for _, d, i, j in ft.ft_wavefront_cells(1, 3, 3, 3)}
     assert len(grid) == 8
+
+
+def _build_c_example(tmp_path):
+    import shutil
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    pkg = os.path.join(root, "paper_conf_sosp_liuqc0hs0y24_b200")
+    out = str(tmp_path / "c_abi_example")
+    if shutil.which("gcc") is None:
+        pytest.skip("gcc not available")
+    subprocess.check_call(["gcc", "-O2", "-I", os.path.join(root, "include"), "-I", "/usr/local/cuda/include",
+                           os.path.join(root, "examples", "c_abi_example.c"), "-L", pkg, "-lft",
+                           "-L", "/usr/local/cuda/lib64", "-lcudart", "-lm", f"-Wl,-rpath,{pkg}", "-o", out])
+    return out
+
+
+def test_c_abi_example_builds_against_the_header(tmp_path):
+    """The C ABI is usable from plain C: examples/c_abi_example.c compiles against include/ft.h
+    and links libft.so (running it needs a GPU: tests/test_gpu_parity.py)."""
+    assert os.path.exists(_build_c_example(tmp_path))

@@ -612,3 +612,15 @@ def test_bf16_grid_depth_bands(B, Lx, Ly, H, D, band, monkeypatch):
     _check(got, ref, torch.bfloat16, keys, ctx=f"grid band {B, Lx, Ly, H, D, band}")
     for k in keys:
         assert torch.equal(got[k], ref_gpu[k]), k
+
+
+def test_c_abi_example_runs(tmp_path):
+    """examples/c_abi_example.c (plain C, no Python in the call path) runs a host-buffer forward
+    and refuses an unsupported shape."""
+    import subprocess
+    from test_abi import _build_c_example
+    exe = _build_c_example(tmp_path)
+    r = subprocess.run([exe, "130", "12", "128", "3"], capture_output=True, text=True, timeout=120)
+    assert r.returncode == 0, r.stdout + r.stderr
+    assert "status OK, finite 1" in r.stdout, r.stdout
+    assert "FT_ERR_UNSUPPORTED" in r.stdout, r.stdout
