@@ -1160,9 +1160,9 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
         if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
         return launch_wavefront_resident(p, t, s, resident_bnu(p, nsm), err);
     }
-    // N-tile width: 64 units by default; 32 units when a diagonal at 64 units cannot give every
-    // CTA group a tile (few cells per diagonal, e.g. the 6-layer dilated C4): twice the tiles, half
-    // the per-tile latency on the dependency chain.
+    // N-tile width: 64 units by default; 32 units only when a diagonal at 64 units would give
+    // under a quarter of the CTA groups a tile: twice the tiles, half the per-tile latency on the
+    // dependency chain, but 1.5x the operand traffic per FLOP.
     const int cg = p.BM == 2 * ROWS ? 2 : 1;
     int dev = 0, nsm = 148;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
@@ -1180,7 +1180,10 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
             if (n > max_cells) max_cells = n;
         }
     }
-    int units = (max_cells * p.naxes * p.MB * p.NT < nsm / cg && p.cell == CELL_LSTM && p.H % 32 == 0) ? 32 : 64;
+    // (round 2: with the leaner epilogue and tile decode, 64-unit tiles beat 32-unit ones on C4
+    //  — 0.902 -> 0.852 ms — although its diagonals give only 48 of 74 CTA pairs a tile; the
+    //  32-unit split now only pays on diagonals a quarter of that wide)
+    int units = (4 * max_cells * p.naxes * p.MB * p.NT < nsm / cg && p.cell == CELL_LSTM && p.H % 32 == 0) ? 32 : 64;
     if (const char* env = getenv("FT_TILE_UNITS")) units = atoi(env) == 32 && p.cell == CELL_LSTM ? 32 : 64;
     if (units == 64)
         return cg == 2 ? launch_cg<2, 64>(p, t, s, err) : launch_cg<1, 64>(p, t, s, err);
