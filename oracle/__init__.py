@@ -5,8 +5,10 @@ import this package.  It wraps the plain-C loop nest in ft_oracle.c (the paper's
 see that file's header for the PAPER.md citations) through ctypes.  It shares no code with the
 CUDA path (paper_conf_sosp_liuqc0hs0y24_b200/) and never imports it.
 
-Pins: tests/test_oracle_pins.py (P1–P12 of SURVEY.md §8(c) c.6).  The grid cell (R12–R14)
-is "parity unpinned" by the paper beyond its Ly=1 / Lx=1 reductions (P8).
+Pins: tests/test_oracle_pins.py (P1–P14 of SURVEY.md §8(c) c.6).  The grid cell (R12–R14)
+is "parity unpinned" by the paper beyond its Ly=1 / Lx=1 reductions (P8): the paper never
+defines it.  The oracle's reading is pinned by P8/P8b, the no-recurrence closed form P8c and
+the exact dependence cone P8d.
 """
 from __future__ import annotations
 

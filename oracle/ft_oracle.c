@@ -18,6 +18,8 @@
  *                   DESIGN.md R12–R14 (Grid LSTM [18], L497): per-axis LSTM transforms sharing
  *                   s = [h^x_{i-1,j}; h^y_{i,j-1}].  PARITY UNPINNED BY THE PAPER beyond the
  *                   Ly=1 / Lx=1 reductions (tests P8) — the paper never defines the grid cell.
+ *                   The reading itself is pinned by P8/P8b (reductions, axis swap), P8c (no
+ *                   recurrence: per-axis batched-matmul closed form) and P8d (dependence cone).
  *
  * Readings of the paper: gate order (i,f,o,ĝ) = gs[0..3] (L611–L615,
  * R1/R2); W multiplies the layer input, U the recurrent h (R3, "x@w + h@u", L609); one bias per

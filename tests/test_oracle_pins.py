@@ -259,6 +259,71 @@ def test_p8b_grid_symmetry_swap_axes():
                                rtol=0, atol=1e-14)
 
 
+def test_p8c_grid_no_recurrence_is_per_axis_batched_matmul():
+    """P8(c) (special case → batched matmul, the grid analogue of P4): U = 0 and both axes'
+    b_f = −40 ⇒ every cell is one LSTM step from the zero state, so with depth 2
+        h^x_0(i,j) = o·tanh(i·ĝ) of x[i]@W[0][x] + b[0][x]   (depends on i only),
+        h^y_0(i,j) = the same of ys[j]@W[0][y] + b[0][y]      (depends on j only),
+        h^a_1(i,j) = the same of h^a_0(i,j)@W[1][a] + b[1][a]  (depth feeds each axis upward).
+    Pins, without the recurrence, which input feeds which axis (R13), which weight slice and
+    bias each axis uses, and the depth wiring of R12 — none of which the Ly = 1 / Lx = 1
+    reductions (P8) can see for the other axis."""
+    B, Lx, Ly, H, D = 2, 3, 4, 8, 2
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, seed=15, dtype="f32", scale=2.0)
+    g["U"][:] = 0
+    g["b"][:, :, 1, :] = -40.0
+    r = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"])
+    W, b = g["W"].astype(np.float64), g["b"].astype(np.float64)
+    sig = lambda v: 1 / (1 + np.exp(-v))
+
+    def step(a, Wg, bg):  # a [..., H] @ Wg [4][H][H] + bg [4][H]
+        z = np.einsum("...k,gkn->...gn", a, Wg) + bg
+        i, o, gg = sig(z[..., 0, :]), sig(z[..., 2, :]), np.tanh(z[..., 3, :])
+        return o * np.tanh(i * gg)
+
+    hx0 = step(g["x"].astype(np.float64), W[0, 0], b[0, 0])   # [B][Lx][H]
+    hy0 = step(g["ys"].astype(np.float64), W[0, 1], b[0, 1])  # [B][Ly][H]
+    hx1 = step(hx0, W[1, 0], b[1, 0])
+    hy1 = step(hy0, W[1, 1], b[1, 1])
+    want = np.empty((B, Lx, Ly, 2, H))
+    want[:, :, :, 0, :] = hx1[:, :, None, :]
+    want[:, :, :, 1, :] = hy1[:, None, :, :]
+    np.testing.assert_allclose(r["out"], want, rtol=0, atol=1e-14)
+
+
+@pytest.mark.parametrize("axis,pos", [(0, 1), (1, 2)])
+def test_p8d_grid_dependence_cone(axis, pos):
+    """P8(d) (invariant): the grid nest's dependence vectors are e_depth, e_x, e_y (Table 4
+    L307–L317 extended to two sequence axes; three nested scans, L421).  Under R12 the input
+    x[i0] enters every cell of row i0 through the x-axis transform only, and the y-axis
+    transform sees row i0 through s = [h^x_{i−1,j}; …] one row later; symmetrically for ys[j0].
+    So perturbing x[i0] changes exactly  out^x at i ≥ i0  and  out^y at i ≥ i0 + 1  (every j),
+    bitwise nothing else; perturbing ys[j0] changes exactly  out^y at j ≥ j0  and  out^x at
+    j ≥ j0 + 1.  A wrong neighbour offset (i+1 for i−1, j for i), an input fed to the wrong
+    axis, or a missing e_x / e_y edge moves a boundary of this pattern."""
+    B, Lx, Ly, H, D = 2, 4, 5, 8, 2
+    g = ftgen.grid_inputs(B, Lx, Ly, H, D, seed=16, dtype="f32", scale=2.0)
+    r = oracle.grid_rnn(g["x"], g["ys"], g["W"], g["U"], g["b"])
+    key = "x" if axis == 0 else "ys"
+    g2 = dict(g)
+    g2[key] = g[key].copy()
+    g2[key][:, pos, :] += 0.5
+    r2 = oracle.grid_rnn(g2["x"], g2["ys"], g2["W"], g2["U"], g2["b"])
+    changed = np.any(r["out"] != r2["out"], axis=-1)  # [B][Lx][Ly][2]
+    i = np.arange(Lx)[:, None]
+    j = np.arange(Ly)[None, :]
+    want = np.zeros((Lx, Ly, 2), bool)
+    if axis == 0:
+        want[..., 0] = np.broadcast_to(i >= pos, (Lx, Ly))
+        want[..., 1] = np.broadcast_to(i >= pos + 1, (Lx, Ly))
+    else:
+        want[..., 1] = np.broadcast_to(j >= pos, (Lx, Ly))
+        want[..., 0] = np.broadcast_to(j >= pos + 1, (Lx, Ly))
+    assert np.array_equal(changed, np.broadcast_to(want, changed.shape))
+    # the final state sits at (Lx−1, Ly−1): inside both axes' cones at every depth
+    assert np.all(np.abs(r["h_n"] - r2["h_n"]).max(axis=-1) > 0)
+
+
 # --------------------------------------------------------------------------- P9
 @pytest.mark.parametrize("beta", [0.4, -1.3])
 def test_p9_saturated_gates(beta):
