@@ -113,9 +113,10 @@ struct WsPlan {
 WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     WsPlan w{};
     w.flags_off = 0;
-    // readiness counters: [2][ncells][MB] (h-ready, c-ready: ft_common.cuh cflag_index), then
-    // ncells * naxes * MB * NT tile counters (tflag_index, the tile-granular protocol)
-    size_t nflags = (2 * (size_t)p.ncells * p.MB + 3) / 4 * 4 + (size_t)p.ncells * p.naxes * p.MB * p.NT;
+    // readiness counters: [2][ncells][MB] (h-ready, c-ready: ft_common.cuh cflag_index), at
+    // least ncells * naxes * MB * NT ints (room for tile-granular protocols)
+    size_t nflags = (size_t)p.ncells * p.naxes * p.MB * p.NT;
+    if (nflags < 2 * (size_t)p.ncells * p.MB) nflags = 2 * (size_t)p.ncells * p.MB;
     w.flags_bytes = round_up(nflags * sizeof(int), 256);
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);

@@ -50,8 +50,6 @@ struct Problem {
     int x_direct;        // bf16 streaming: layer-0 inputs read from x [B][T][H] (host-IO overlap)
     int owner;           // KIND_SEQ tile assignment (see TileWalk): 0 round-robin, 1 owner-computes
                          // under bands, 2 layer 0 owned (dilated nests) + round-robin for the rest
-    int tiledep;         // owner walk, 64-unit tiles: activation chunk kc waits on the producer's
-                         // N-tile kc counter (tflag_index) instead of its whole-cell counter
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
@@ -209,13 +207,6 @@ FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
 // the h-ready counter covers both.
 FT_HD long long cflag_index(const Problem& p, long long cell, int m) {
     return (p.ncells + cell) * p.MB + m;
-}
-
-// Tile counters of P.tiledep, after the h-ready and c-ready counters: one per (cell, m-block,
-// N-tile), complete at flag_mult (every epilogue warp of the tile's CTAs increments once).
-// The region starts 16-byte aligned, so a cell's NT (a multiple of 4) counters load as int4s.
-FT_HD long long tflag_index(const Problem& p, long long cell, int m, int n) {
-    return (2 * p.ncells * p.MB + 3) / 4 * 4 + (cell * p.MB + m) * (long long)p.NT + n;
 }
 
 // Tile-granular protocol of the bf16 streaming kernel: one counter per (cell, axis, m-block,
@@ -591,10 +582,6 @@ __device__ __forceinline__ void red_release_gpu_add(int* p, int v) {
     asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-__device__ __forceinline__ void red_relaxed_gpu_add(int* p, int v) {
-    asm volatile("red.relaxed.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
 __device__ __forceinline__ void fence_acq_rel_sys() {
     asm volatile("fence.acq_rel.sys;" ::: "memory");
 }
@@ -616,23 +603,6 @@ __device__ __forceinline__ void wait_flag_geq_sys(const int* p, int target) {
         if (ld_acquire_sys(p) >= target) return;
         if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
     }
-}
-
-// Tile counters of one producer cell (P.tiledep == 2): nt (a multiple of 4, at most 32)
-// consecutive 16-byte-aligned counters read with relaxed vector loads, all in flight at once;
-// returns the mask of those at >= target.  Callers follow a hit with fence_acq_rel_gpu()
-// (fence-based acquire).
-__device__ __forceinline__ uint32_t tile_ready_mask(const int* p, int nt, int target) {
-    uint32_t m = 0;
-#pragma unroll 1
-    for (int n = 0; n < nt; n += 4) {
-        int a, b, c, d;
-        asm volatile("ld.relaxed.gpu.global.v4.s32 {%0, %1, %2, %3}, [%4];"
-                     : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "l"(p + n) : "memory");
-        m |= (uint32_t)(a >= target) << n | (uint32_t)(b >= target) << (n + 1) |
-             (uint32_t)(c >= target) << (n + 2) | (uint32_t)(d >= target) << (n + 3);
-    }
-    return m;
 }
 
 // Bounded acquire-spin on a readiness counter.

@@ -222,8 +222,6 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const bool skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
     const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : CG * C::A_BYTES;
     TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
-    const bool tdep = !kWeights && U == 64 && P.tiledep && P.owner == 1;
-    uint32_t rmask = 0;  // P.tiledep == 2: producer N-tiles of the current segment known ready
     FT_TR_ROLE;
     TileId tl;
     long long tile;
@@ -247,25 +245,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                 // the segment's producer cell (Table 4 dependence vectors): one acquire of its
                 // (cell, m-block) counter before the segment's first activation load, so inputs
                 // that are ready (x, the layer below) stream in while a later producer finishes
-                if (tdep && sg.scell >= 0 && !(P.debug & 1)) {
-                    // tile-granular: K chunk kc of a 64-unit producer is its N-tile kc
-                    FT_TR_BEGIN();
-                    if (P.tiledep == 2) {  // batched polls: one round trip covers every N-tile
-                        if (kc == 0) rmask = 0;
-                        if (!((rmask >> kc) & 1)) {
-                            const int* base = T.flags + tflag_index(P, sg.scell, tl.m, 0);
-                            const uint64_t t0 = globaltimer_ns();
-                            while (!(((rmask = tile_ready_mask(base, P.NT, P.flag_mult)) >> kc) & 1))
-                                if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
-                            fence_acq_rel_gpu();
-                        }
-                    } else {
-                        wait_flag_geq(T.flags + tflag_index(P, sg.scell, tl.m, kc), P.flag_mult);
-                    }
-                    FT_TR_END(TR_P_FLAG);
-                    if (kc == 0 && rank == 0) FT_EV(tile, 5);
-                    fence_proxy_async_global();
-                } else if (kc == 0 && sg.scell >= 0 && !(P.debug & 1)) {
+                if (kc == 0 && sg.scell >= 0 && !(P.debug & 1)) {
                     FT_TR_BEGIN();
                     wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
                     FT_TR_END(TR_P_FLAG);
@@ -515,7 +495,6 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
     const bool own = P.owner == 1 || (P.owner == 2 && (int)(blockIdx.x / CG) < P.NT);
     const bool split = P.band > 0 && !own;
-    const bool tdep_rel = U == 64 && P.tiledep && P.owner == 1;
     float cst[EPI_UNITS];
 #pragma unroll
     for (int v = 0; v < EPI_UNITS; ++v) cst[v] = 0.f;
@@ -693,8 +672,6 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 __nanosleep(200 + (h & 4095u));
             }
             red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
-            // tile counter: ordered after the release's fence, so it publishes the same stores
-            if (tdep_rel) red_relaxed_gpu_add(T.flags + tflag_index(P, cell_lin(P, c.d, c.i, c.j), tl.m, tl.n), 1);
         }
         if (leader_thread) {
             FT_TR_END(TR_E_WORK);
@@ -1094,9 +1071,6 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         q.owner = unit_dil && p.MB == 1 && p.naxes == 1 && (long long)q.band * p.NT <= grid / CG;
         if (const char* e = getenv("FT_OWNER")) q.owner = q.owner && atoi(e) != 0;  // A/B
         if (const char* e = getenv("FT_SKEW")) q.skew = atoi(e);
-        if (const char* e = getenv("FT_TILEDEP"))  // A/B: 1 per-chunk acquire, 2 batched polls
-            q.tiledep = (q.owner == 1 && (atoi(e) == 1 || (atoi(e) == 2 && p.NT % 4 == 0 && p.NT <= 32)))
-                            ? atoi(e) : 0;
     }
     cudaLaunchAttribute attr2[2];
     if (q.band == 0 && p.resident_layers == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM &&

@@ -544,33 +544,6 @@ def test_bf16_layer_bands_stress(monkeypatch):
     _check(first, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="band stress")
 
 
-@pytest.mark.parametrize("mode", ["1", "2"])
-@pytest.mark.parametrize("B,T,H,D,band,debug", [
-    (256, 6, 256, 6, 4, "0"),    # tile counters, short last band
-    (256, 5, 256, 5, 2, "64"),   # stress mode: random delays before every counter release
-    (130, 4, 512, 4, 2, "0"),    # padded batch rows in the CTA pair, 8 N-tiles
-])
-def test_bf16_owner_tile_counters(mode, B, T, H, D, band, debug, monkeypatch):
-    """Tile-granular dependencies under the owner walk (FT_TILEDEP=1: one acquire per K chunk;
-    2: batched relaxed polls of a producer cell's tile counters + fence-based acquire): each
-    activation K chunk waits on its producer N-tile's counter instead of the whole cell's.
-    Outputs against the oracle, and bitwise equal to the paper order (same per-cell
-    arithmetic, finer waits)."""
-    monkeypatch.setenv("FT_RESIDENT", "0")
-    monkeypatch.setenv("FT_TILE_UNITS", "64")  # tile counters need 64-unit tiles (chunk = tile)
-    p = ftgen.stacked_inputs(B, T, H, D, 1919 + band, "bf16")
-    monkeypatch.setenv("FT_BAND", "0")
-    ref_gpu = _run_stacked(p, torch.bfloat16, want_all=True)
-    monkeypatch.setenv("FT_BAND", str(band))
-    monkeypatch.setenv("FT_TILEDEP", mode)
-    monkeypatch.setenv("FT_DEBUG", debug)
-    for _ in range(2):
-        got = _run_stacked(p, torch.bfloat16, want_all=True)
-        for k in ALL:
-            assert torch.equal(got[k], ref_gpu[k]), f"{k}: tile counters not bitwise equal to the paper order"
-    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"tiledep {B,T,H,D,band}")
-
-
 # ------------------------------------------------------------------------- host-buffer call (e2e)
 @pytest.mark.parametrize("B,T,H,D,env", [
     (256, 23, 128, 6, {"FT_BAND": "2", "FT_RESIDENT": "0"}),                  # bands, owner walk
