@@ -40,5 +40,32 @@ xs = torch.from_numpy(p["x"]).to(dev, torch.bfloat16)     # NEXT-3 linear RNN
 ft.stacked_rnn(xs, a[1][:, 0].contiguous())
 g = ftgen.b2b_inputs(256, 256, 64, 64, 1, "bf16")          # NEXT-4 back-to-back GEMMs
 ft.b2b_gemm(*[torch.from_numpy(g[k]).to(dev, torch.bfloat16) for k in ("A", "B", "C")])
+# round 2b features
+os.environ["FT_CLUSTER"] = "1"                            # DSMEM cluster kernel (C2 class)
+run_seq(37, 5, 128, 3, torch.bfloat16)
+os.environ.pop("FT_CLUSTER")
+run_seq(256, 6, 128, 6, torch.bfloat16, dil=[1, 2, 4, 1, 2, 4], resident="0")  # dilated, x read in place
+os.environ["FT_OWNER_L0"] = "1"                           # layer-0 owners (dilated)
+run_seq(256, 6, 128, 4, torch.bfloat16, dil=[1, 2, 3, 4], resident="0")
+os.environ.pop("FT_OWNER_L0")
+os.environ["FT_BAND"] = "2"                               # grid depth bands
+run_grid(130, 3, 4, 128, 4, torch.bfloat16)
+os.environ.update(FT_RESIDENT="0")                        # host-buffer call under bands (x/y overlap)
+B, T, H, D = 256, 12, 128, 6
+p = ftgen.stacked_inputs(B, T, H, D, 1, "bf16")
+W, U = (torch.from_numpy(p[k]).to(dev, torch.bfloat16) for k in ("W", "U"))
+bb = torch.from_numpy(p["b"]).to(dev)
+x_h = torch.from_numpy(p["x"]).to(torch.bfloat16).pin_memory()
+y_h = torch.empty((B, T, H), dtype=torch.bfloat16).pin_memory()
+hn_h = torch.empty((B, D, H), dtype=torch.bfloat16).pin_memory()
+cn_h = torch.empty((B, D, H), dtype=torch.float32).pin_memory()
+nb = ft.ft_stacked_lstm_hostio_workspace_size(B, T, H, D, ft.FT_BF16)
+ws = torch.empty(nb, dtype=torch.uint8, device=dev)
+s = torch.cuda.Stream()
+ft.check(ft.ft_stacked_lstm_fwd_hostio(B, T, H, D, ft.FT_BF16, x_h.data_ptr(), W.data_ptr(), U.data_ptr(),
+                                       bb.data_ptr(), y_h.data_ptr(), hn_h.data_ptr(), cn_h.data_ptr(),
+                                       ws.data_ptr(), nb, s.cuda_stream))
+s.synchronize()
+os.environ.pop("FT_BAND")
 torch.cuda.synchronize()
 print("sanitize cases done")
