@@ -125,7 +125,11 @@ struct KCfg {
     static constexpr uint32_t IDESC = make_idesc_bf16_f32(ROWS * CG, BN, false, true);
     static constexpr int EPI_UNITS = U / EPI_PARTS;            // units per epilogue thread
     // units per TMEM load: 16, or 8 with 16 epilogue warps (register budget of 608 threads)
+#ifdef FT_EPI_CH  // experiments: 8 or 16
+    static constexpr int EPI_CH = EPI_UNITS < FT_EPI_CH ? EPI_UNITS : FT_EPI_CH;
+#else
     static constexpr int EPI_CH = EPI_UNITS < 16 / EPI_PARTS * 2 ? EPI_UNITS : 16 / EPI_PARTS * 2;
+#endif
 };
 
 struct Maps {
