@@ -610,9 +610,19 @@ __device__ __forceinline__ void wait_flag_geq(const int* p, int target) {
     if (ld_acquire_gpu(p) >= target) return;
     const uint64_t t0 = globaltimer_ns();
     for (;;) {
+#ifdef FT_POLL_RELAXED  // experiment: spin on relaxed loads (no L1 invalidate per poll), then
+                        // one acquire load of the (monotone) counter once it is there
+#pragma unroll 1
+        for (int it = 0; it < 256; ++it)
+            if (ld_relaxed_gpu(p) >= target) {
+                (void)ld_acquire_gpu(p);
+                return;
+            }
+#else
 #pragma unroll 1
         for (int it = 0; it < 256; ++it)
             if (ld_acquire_gpu(p) >= target) return;
+#endif
         if (globaltimer_ns() - t0 > FT_SPIN_TIMEOUT_NS) __trap();
     }
 }
