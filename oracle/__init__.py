@@ -35,24 +35,62 @@ def build(force: bool = False) -> str:
     return LIB_PATH
 
 
-_lib = None
+def _host_key() -> str:
+    """Identifies the host CPU, so a -march=native build is never loaded on another CPU model."""
+    import hashlib
+    model = ""
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                if line.startswith(("model name", "flags")):
+                    model += line
+                    if line.startswith("flags"):
+                        break
+    except OSError:
+        pass
+    return hashlib.sha1(model.encode()).hexdigest()[:12]
 
 
-def lib():
-    global _lib
-    if _lib is None:
-        build()
-        _lib = ctypes.CDLL(LIB_PATH)
+def timing_lib_path() -> str:
+    return os.path.join(_HERE, f"liboracle_timing_{_host_key()}.so")
+
+
+def build_timing(force: bool = False) -> str:
+    """The CPU-baseline build of the SAME source: -O3 -march=native for the
+    host it runs on, still -ffp-contract=off and no -ffast-math, so every output is bitwise the
+    parity build's (pinned in tests/test_oracle_pins.py).  Compiled on first use on each host
+    (the GPU box's CPU may differ from the build machine's)."""
+    path = timing_lib_path()
+    newest = max(os.path.getmtime(s) for s in _SOURCES)
+    if not force and os.path.exists(path) and os.path.getmtime(path) >= newest:
+        return path
+    cmd = ["gcc", "-O3", "-march=native", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+           "-fvisibility=hidden", "-ffp-contract=off", "-o", path + ".tmp", _SOURCES[0], "-lm"]
+    subprocess.check_call(cmd, cwd=_HERE)
+    os.replace(path + ".tmp", path)
+    return path
+
+
+_libs = {}
+
+
+def lib(which: str = "parity"):
+    """The oracle library: "parity" (-O2, portable; the tests' reference) or "timing" (the
+    CPU-baseline build of the same source, bitwise identical results)."""
+    if which not in _libs:
+        path = build() if which == "parity" else build_timing()
+        L = ctypes.CDLL(path)
         for sfx in ("f64", "f32", "bf16emu"):
             for name in ("stacked_lstm", "dilated_rnn", "grid_rnn", "lstm_cell", "stacked_rnn",
                          "b2b_gemm"):
-                fn = getattr(_lib, f"ft_oracle_{name}_{sfx}")
+                fn = getattr(L, f"ft_oracle_{name}_{sfx}")
                 fn.restype = ctypes.c_int if name != "lstm_cell" else None
-    return _lib
+        _libs[which] = L
+    return _libs[which]
 
 
-def num_threads() -> int:
-    return int(lib().ft_oracle_num_threads())
+def num_threads(which: str = "parity") -> int:
+    return int(lib(which).ft_oracle_num_threads())
 
 
 def _p(a):
@@ -71,7 +109,7 @@ def _c(a, dt):
     return np.ascontiguousarray(a, dtype=dt)
 
 
-def stacked_lstm(x, W, U, b, precision="f64", want_all=False):
+def stacked_lstm(x, W, U, b, precision="f64", want_all=False, build_kind="parity"):
     """Stacked LSTM oracle (Listing 2).  x [B][T][H], W/U [D][4][H][H], b [D][4][H]."""
     dt = _prec(precision)
     B, T, H = x.shape
@@ -82,7 +120,7 @@ def stacked_lstm(x, W, U, b, precision="f64", want_all=False):
     c_n = np.empty((B, D, H), dt)
     h_all = np.empty((B, D, T, H), dt) if want_all else None
     c_all = np.empty((B, D, T, H), dt) if want_all else None
-    rc = getattr(lib(), f"ft_oracle_stacked_lstm_{precision}")(
+    rc = getattr(lib(build_kind), f"ft_oracle_stacked_lstm_{precision}")(
         B, T, H, D, _p(x), _p(W), _p(U), _p(b), _p(y), _p(h_n), _p(c_n), _p(h_all), _p(c_all))
     if rc:
         raise RuntimeError(f"oracle stacked_lstm failed: {rc}")

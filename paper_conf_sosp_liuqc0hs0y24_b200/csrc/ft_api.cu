@@ -72,12 +72,16 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
                 : (double)D * p->naxes * 4.0 * H * ((double)H + (kind == ft::KIND_SEQ ? H : 2.0 * H)) *
                       (dt == FT_BF16 ? 2 : 4);
         p->resident_layers = wbytes <= 64.0 * 1024 * 1024 ? D : 0;
-        const char* env = getenv("FT_L2_RESIDENT_LAYERS");  // tuning override
-        if (env) p->resident_layers = atoi(env);
-        const char* pe = getenv("FT_L2_PERSIST_LAYERS");  // experiments: force the window's layer count
-        p->persist_layers = pe ? atoi(pe) : -1;            // -1: sized by ft_set_l2_persist (auto)
-        const char* dbg = getenv("FT_DEBUG");  // timing experiments only
-        p->debug = dbg ? atoi(dbg) : 0;
+        p->persist_layers = -1;  // -1: sized by ft_set_l2_persist
+        p->debug = 0;
+#ifdef FT_DEV_EXPERIMENTS  // development builds only (tools/variant_build.sh); never in libft.so
+        if (const char* env = getenv("FT_L2_RESIDENT_LAYERS")) p->resident_layers = atoi(env);
+        if (const char* pe = getenv("FT_L2_PERSIST_LAYERS")) p->persist_layers = atoi(pe);
+        if (const char* dbg = getenv("FT_DEBUG")) p->debug = atoi(dbg);  // results INVALID
+#endif
+        // documented schedule knob (include/ft.h): random delays before every counter release;
+        // results are unchanged, the tests use it to shake out ordering bugs
+        if (ft::env_flag("FT_STRESS")) p->debug |= 64;
     }
     p->BNU = dt == FT_BF16 ? ft::BF16_BNU : ft::F32_BNU;
     if (cell == ft::CELL_LINEAR && dt == FT_BF16) p->BNU = 4 * ft::BF16_BNU;  // 256 units per tile
@@ -113,10 +117,8 @@ struct WsPlan {
 WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     WsPlan w{};
     w.flags_off = 0;
-    // readiness counters: [2][ncells][MB] (h-ready, c-ready: ft_common.cuh cflag_index), at
-    // least ncells * naxes * MB * NT ints (room for tile-granular protocols)
-    size_t nflags = (size_t)p.ncells * p.naxes * p.MB * p.NT;
-    if (nflags < 2 * (size_t)p.ncells * p.MB) nflags = 2 * (size_t)p.ncells * p.MB;
+    // readiness counters: [2][ncells][MB] (h-ready, c-ready: ft_common.cuh cflag_index)
+    const size_t nflags = 2 * (size_t)p.ncells * p.MB;
     w.flags_bytes = round_up(nflags * sizeof(int), 256);
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
@@ -149,6 +151,50 @@ ft_status check_device() {
     return FT_OK;
 }
 
+// Co-residency of persistent launches.  The wavefront kernels spin on each other's CTAs, so all
+// CTAs of one launch must be resident together.  A single launch guarantees that by construction
+// (cooperative launch, or a cluster grid sized by cudaOccupancyMaxActiveClusters), but two of the
+// library's launches on two streams of one device could split the SMs between them and both spin.
+// So every persistent launch of this process on a device is ordered after the previous one: the
+// caller's stream waits on an event recorded after the previous launch (no host blocking; the
+// streams stay otherwise independent).  Skipped while the stream is being captured into a graph
+// (the graph's own launch order applies).  Processes without MPS never run kernels concurrently.
+class PersistentOrder {
+  public:
+    explicit PersistentOrder(cudaStream_t s) : s_(s) {
+        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing(s, &cs) != cudaSuccess) {
+            cudaGetLastError();
+            return;
+        }
+        if (cs != cudaStreamCaptureStatusNone) return;
+        int dev = 0;
+        if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return;
+        lock_ = std::unique_lock<std::mutex>(mu());
+        cudaEvent_t& ev = last()[dev];
+        if (!ev && cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) {
+            cudaGetLastError();
+            ev = nullptr;
+            lock_.unlock();
+            return;
+        }
+        ev_ = ev;
+        if (used()[dev] && cudaStreamWaitEvent(s, ev, 0) != cudaSuccess) cudaGetLastError();
+        used()[dev] = true;
+    }
+    ~PersistentOrder() {
+        if (ev_ && cudaEventRecord(ev_, s_) != cudaSuccess) cudaGetLastError();
+    }
+
+  private:
+    static std::mutex& mu() { static std::mutex m; return m; }
+    static cudaEvent_t* last() { static cudaEvent_t e[64] = {}; return e; }
+    static bool* used() { static bool u[64] = {}; return u; }
+    cudaStream_t s_;
+    cudaEvent_t ev_ = nullptr;
+    std::unique_lock<std::mutex> lock_;
+};
+
 ft_status run(const ft::Problem& p, ft_dtype dt, ft::Tensors t, void* workspace,
               size_t workspace_bytes, void* stream) {
     const WsPlan w = plan_workspace(p, dt, t.h_all != nullptr);
@@ -171,6 +217,7 @@ ft_status run(const ft::Problem& p, ft_dtype dt, ft::Tensors t, void* workspace,
     } else if (!t.h_all)
         t.h_all = ws + w.hall_off;
     cudaStream_t s = static_cast<cudaStream_t>(stream);
+    PersistentOrder order(s);
     cudaError_t e = cudaMemsetAsync(t.flags, 0, w.flags_bytes, s);  // BK0: reset readiness flags
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("flag reset: ") + cudaGetErrorString(e));
     std::string err;
@@ -224,7 +271,7 @@ ft_status seq_fwd(int batch, int seq, int hidden, int depth, const int* dil, ft_
 }  // namespace
 
 namespace ft {
-static int g_l2_persist_mib = -1;  // ft_set_l2_persist: -1 auto, 0 off, else MiB
+static int g_l2_persist_mib = 0;  // ft_set_l2_persist: 0 off (default), -1 auto, else MiB
 int l2_persist_mib() { return g_l2_persist_mib; }
 void set_last_error(const std::string& msg) { g_last_error = msg; }
 long long c_ring_elems(const Problem& p) {
@@ -542,6 +589,7 @@ FT_API ft_status ft_stacked_lstm_layerwise_fwd(int batch, int seq, int hidden, i
     std::string why;
     if (ft::layerwise_supported(batch, hidden, nsm, &why) != 0) return fail(FT_ERR_UNSUPPORTED, why);
     std::string err;
+    PersistentOrder order(static_cast<cudaStream_t>(stream));
     cudaError_t e = ft::launch_layerwise(batch, seq, hidden, depth, x, W, U, b, y, h_n, c_n, h_all,
                                          c_all, workspace, static_cast<cudaStream_t>(stream), &err);
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, err.empty() ? cudaGetErrorString(e) : err);

@@ -14,6 +14,15 @@
 
 #include "../../include/ft.h"
 
+// Result-invalidating timing experiments (FT_DEBUG bits other than the stress bit 64) exist only
+// in development builds compiled with -DFT_DEV_EXPERIMENTS; in the release library the test is a
+// compile-time false, so no such branch is even in the binary.
+#ifdef FT_DEV_EXPERIMENTS
+#define FT_DEV_BIT(dbg, bit) (((dbg) & (bit)) != 0)
+#else
+#define FT_DEV_BIT(dbg, bit) false
+#endif
+
 #ifdef __CUDACC__
 #define FT_HD __host__ __device__ __forceinline__
 #else
@@ -40,11 +49,12 @@ struct Problem {
     int resident_layers; // bf16: layers whose weights are kept in L2 (evict_last); others stream
     int persist_layers;  // bf16 streaming: W of the first persist_layers layers lie in a persisting
                          // L2 access-policy window (loaded with EVICT_NORMAL); host side: -1 = auto
-    int debug;           // timing experiments only (env FT_DEBUG; results invalid when != 0):
-                         // 1 skip dependency waits, 2 skip the epilogue math/stores, 4 no MMAs,
-                         // 16 no weight loads, 32 fixed load coordinates, 128 EVICT_NORMAL state;
-                         // 64 = stress mode: random delays before each counter release
-                         // (results stay valid; used by tests to shake out ordering bugs)
+    int debug;           // 64 = stress mode (env FT_STRESS=1): random delays before each counter
+                         // release — results stay valid; tests use it to shake out ordering bugs.
+                         // Development builds only (-DFT_DEV_EXPERIMENTS, env FT_DEBUG; never
+                         // compiled into libft.so, results INVALID): 1 skip dependency waits,
+                         // 2 skip the epilogue math/stores, 4 no MMAs, 16 no weight loads,
+                         // 32 fixed load coordinates, 128 EVICT_NORMAL state
     int l2pol;           // bf16 streaming: L2 eviction-policy overrides, 2 bits each (0 default,
                          // 1 first, 2 normal, 3 last): weights | state stores << 2 | A loads << 4
     int x_direct;        // bf16 streaming: layer-0 inputs read from x [B][T][H] (host-IO overlap)
@@ -207,14 +217,6 @@ FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
 // the h-ready counter covers both.
 FT_HD long long cflag_index(const Problem& p, long long cell, int m) {
     return (p.ncells + cell) * p.MB + m;
-}
-
-// Tile-granular protocol of the bf16 streaming kernel: one counter per (cell, axis, m-block,
-// N-tile), complete when it reaches flag_mult (the CTAs of the tile).  A consumer's K-chunk kc
-// only needs the producer's units [kc*64, kc*64+64) — one N-tile — so consecutive diagonals
-// pipeline at tile granularity instead of waiting for whole cells.
-FT_HD long long tile_flag(const Problem& p, long long cell, int axis, int m, int n) {
-    return ((cell * p.naxes + axis) * p.MB + m) * (long long)p.NT + n;
 }
 
 // Monotone cursor over the tile sequence (tile = cell_ordinal * tiles_per_cell + w).  Every

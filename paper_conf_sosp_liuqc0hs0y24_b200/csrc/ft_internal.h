@@ -3,11 +3,21 @@
 
 #include <cuda_runtime.h>
 
+#include <cstdlib>
 #include <string>
+#include <utility>
 
 #include "ft_common.cuh"
 
 namespace ft {
+
+// Environment knobs (every one is documented in include/ft.h; none changes a result beyond the
+// summation-order freedom that header states).  Read per call, so a test can flip them.
+inline const char* env_str(const char* name) { return getenv(name); }
+inline bool env_flag(const char* name) {  // set and not "0"
+    const char* e = getenv(name);
+    return e && e[0] && !(e[0] == '0' && e[1] == 0);
+}
 
 // Device pointers of one call.  `y` is `out` for the grid call.
 struct Tensors {
@@ -41,6 +51,35 @@ struct Tensors {
     int* ysig_per_chunk = nullptr; // HOST: 1 = owner walk: each warp signals once per chunk (its
                                    // last step of the chunk), so a chunk completes at per_step
 };
+
+// Persistent cluster launch: a cluster grid sized by cudaOccupancyMaxActiveClusters fits the idle
+// device, and the cooperative attribute is added as well when the driver accepts it next to the
+// cluster dimension (remembered per kernel), so the launch fails up front instead of spinning if
+// the grid cannot be co-resident.  Launches of the library on one device are additionally
+// ordered one after another (ft_api.cu PersistentOrder).
+template <typename... KArgs, typename... Args>
+cudaError_t launch_cluster_persistent(cudaLaunchConfig_t cfg, const cudaLaunchAttribute* base, int nbase,
+                                      void (*kernel)(KArgs...), Args&&... args) {
+    static int mode = 0;  // 0 untried, 1 cooperative + cluster accepted, 2 rejected
+    cudaLaunchAttribute a[4];
+    for (int i = 0; i < nbase && i < 3; ++i) a[i] = base[i];
+    if (mode != 2) {
+        a[nbase].id = cudaLaunchAttributeCooperative;
+        a[nbase].val.cooperative = 1;
+        cfg.attrs = a;
+        cfg.numAttrs = nbase + 1;
+        const cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+        if (e == cudaSuccess || mode == 1 || e == cudaErrorCooperativeLaunchTooLarge) {
+            if (e == cudaSuccess) mode = 1;
+            return e;
+        }
+        cudaGetLastError();  // the combination is not supported here: plain cluster launch
+        mode = 2;
+    }
+    cfg.attrs = a;
+    cfg.numAttrs = nbase;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
 
 // Tile shapes of the two kernels.
 constexpr int F32_BM = 32, F32_BNU = 32;     // SIMT correctness path (BK1)

@@ -48,7 +48,8 @@ constexpr uint32_t LIDESC = make_idesc_bf16_f32(LROWS, LN, false, true);
 struct LayerArgs {
     int B, T, H, D, d, MB, NTR;
     int stages;            // A ring depth (shared memory left after the U slab)
-    int debug;             // FT_DEBUG timing experiments: 8 = skip the A loads (wrong results)
+    int debug;             // development builds only (FT_DEV_EXPERIMENTS, env FT_DEBUG): 8 = skip
+                           // the A loads (wrong results); always 0 in libft.so
     int a_rows;            // rows per A box: min(128, batch rounded up to 8) — no padded-row loads
     const float* Z;        // [B][T][4H] fp32 = X_{d-1} @ W_d (gate-major columns)
     const float* b;        // [4][H] bias of layer d
@@ -139,7 +140,7 @@ layer_recurrent_kernel(const __grid_constant__ LayerArgs A, const __grid_constan
                 fence_proxy_async_global();
                 for (int kc = 0; kc < KCH; ++kc) {
                     mbar_wait(&empty[stage], phase ^ 1);
-                    if (A.debug & 8) {
+                    if (FT_DEV_BIT(A.debug, 8)) {
                         mbar_arrive(&full[stage]);
                         if (++stage == S) {
                             stage = 0;
@@ -511,7 +512,11 @@ cudaError_t launch_layerwise(int B, int T, int H, int D, const void* x, const vo
         a.MB = MB;
         a.NTR = NTR;
         a.stages = stages;
+#ifdef FT_DEV_EXPERIMENTS  // development builds only (tools/variant_build.sh); never in libft.so
         a.debug = getenv("FT_DEBUG") ? atoi(getenv("FT_DEBUG")) : 0;
+#else
+        a.debug = 0;
+#endif
         a.a_rows = a_rows;
         a.Z = Z;
         a.b = b + (size_t)d * 4 * H;

@@ -45,6 +45,8 @@
 
 #include <cstdio>
 #include <cstdlib>
+#include <cstring>
+#include <mutex>
 #include <string>
 
 #include "ft_internal.h"
@@ -223,7 +225,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     uint64_t pol_keep = policy_evict_last();
     const uint64_t pol_act = l2_policy((P.l2pol >> 4) & 3, policy_evict_normal());
     if (P.l2pol & 3) pol_stream = pol_keep = l2_policy(P.l2pol & 3, pol_keep);
-    const bool skipB = P.debug & 16, fixed = P.debug & 32;  // timing experiments
+    const bool skipB = FT_DEV_BIT(P.debug, 16), fixed = FT_DEV_BIT(P.debug, 32);  // timing experiments
     const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : CG * C::A_BYTES;
     TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     FT_TR_ROLE;
@@ -249,7 +251,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                 // the segment's producer cell (Table 4 dependence vectors): one acquire of its
                 // (cell, m-block) counter before the segment's first activation load, so inputs
                 // that are ready (x, the layer below) stream in while a later producer finishes
-                if (kc == 0 && sg.scell >= 0 && !(P.debug & 1)) {
+                if (kc == 0 && sg.scell >= 0 && !FT_DEV_BIT(P.debug, 1)) {
                     FT_TR_BEGIN();
                     wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
                     FT_TR_END(TR_P_FLAG);
@@ -327,7 +329,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
             FT_TR_END(TR_M_FULL);
             tc_fence_after();
             if (elect_one()) {
-                if (P.debug & 4) {  // timing experiment: no MMA, hand the slot straight back
+                if (FT_DEV_BIT(P.debug, 4)) {  // timing experiment: no MMA, hand the slot straight back
                     if constexpr (CG == 1) {
                         mbar_arrive(&empty[stage]);
                     } else {
@@ -352,7 +354,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
         }
         if ((threadIdx.x & 31) == 0) FT_EV(tile, 7);
         if (elect_one()) {
-            if (P.debug & 4) {
+            if (FT_DEV_BIT(P.debug, 4)) {
                 if constexpr (CG == 1) {
                     mbar_arrive(&tfull[acc]);
                 } else {
@@ -491,9 +493,9 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     // L2 priority of the nest's live state (the c ring and the blocked h): EVICT_LAST, so the
     // EVICT_FIRST weight stream does not push it out before the next diagonal reads it (ncu, C3:
-    // DRAM 30.8 -> 30.1 GB per launch).  FT_DEBUG bit 128 reverts to EVICT_NORMAL (A/B runs).
+    // DRAM 30.8 -> 30.1 GB per launch).  FT_DEBUG bit 128 (development builds) reverts to EVICT_NORMAL.
     const uint64_t pol_state = l2_policy((P.l2pol >> 2) & 3,
-                                         (P.debug & 128) ? policy_evict_normal() : policy_evict_last());
+                                         FT_DEV_BIT(P.debug, 128) ? policy_evict_normal() : policy_evict_last());
     // owner-computes (TileWalk): this thread's rows x units of the slab are the same in every
     // tile, so the cell state stays in registers (cst) from step t to t + 1 — no c ring, no
     // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
@@ -533,7 +535,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         // (1) the previous cell state, prefetched while this tile's MMAs still run: one acquire
         //     of the c-producer's counter, published to the other epilogue threads by bar.sync
         FT_TR_BEGIN();
-        if (cprod >= 0 && leader_thread && !own && !(P.debug & 1))
+        if (cprod >= 0 && leader_thread && !own && !FT_DEV_BIT(P.debug, 1))
             wait_flag_geq(T.flags + (split ? cflag_index(P, cprod, tl.m) : cprod * P.MB + tl.m), target);
         named_bar_sync(1, EPI_THREADS);
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
@@ -597,7 +599,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                         mbar_arrive_remote_cta(mapa_shared(smem_u32(&tempty[acc]), 0));
                 }
             }
-            if (P.debug & 2) continue;
+            if (FT_DEV_BIT(P.debug, 2)) continue;
             const int ub = half * EPI_UNITS + u0;  // unit offset inside the tile
             float bi[CH], bf[CH], bo[CH], bg[CH];
 #pragma unroll
@@ -671,7 +673,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         _e1 = clock64();
 #endif
         if (lane == 0) {
-            if (P.debug & 64) {  // stress mode (tests): a pseudo-random delay before publishing
+            if (P.debug & 64) {  // stress mode (FT_STRESS=1) (tests): a pseudo-random delay before publishing
                 const uint32_t h = (uint32_t)(tile * 2654435761u) ^ (uint32_t)(blockIdx.x * 40503u + warp * 977u);
                 __nanosleep(200 + (h & 4095u));
             }
@@ -733,7 +735,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         }
         // (4) host-IO overlap: this warp's share of y(·, t, ·) is stored → fence at system scope
         //     (a copy engine reads it) and count it for the copy stream (ft_api.cu hostio)
-        if (top && T.ysig && (!own || c.i % T.ychunk == T.ychunk - 1 || c.i == P.L0 - 1)) {
+        if (top && T.ysig && (P.owner != 1 || c.i % T.ychunk == T.ychunk - 1 || c.i == P.L0 - 1)) {
             // (owner walk: the same warps store every step of their slab, so one fence at the
             //  chunk's last step covers the chunk)
             __syncwarp();
@@ -933,12 +935,48 @@ int choose_band(const Problem& p, int workers) {
     return band;
 }
 
+// Host-side launch state cached across calls (serving loops call the same shapes with the same
+// buffers over and over): the tensor maps per (buffers, shape), and per device the dynamic
+// shared-memory attribute and the cluster occupancy.  Keys hold every input of the encoding, so
+// a hit returns exactly what a fresh encode would.
+struct MapsKey {
+    const void *x, *ys, *W, *U, *hb, *xb, *yb;
+    int kind, cell, B, L0, L1, H, D, MB, BM, x_direct, cg, units, dev;
+    bool operator==(const MapsKey& o) const { return std::memcmp(this, &o, sizeof(MapsKey)) == 0; }
+};
+struct MapsCache {
+    static constexpr int N = 8;
+    std::mutex mu;
+    MapsKey key[N];
+    Maps maps[N];
+    int used = 0, next = 0;
+    bool find(const MapsKey& k, Maps* out) {
+        std::lock_guard<std::mutex> g(mu);
+        for (int i = 0; i < used; ++i)
+            if (key[i] == k) {
+                *out = maps[i];
+                return true;
+            }
+        return false;
+    }
+    void put(const MapsKey& k, const Maps& m) {
+        std::lock_guard<std::mutex> g(mu);
+        key[next] = k;
+        maps[next] = m;
+        next = (next + 1) % N;
+        if (used < N) ++used;
+    }
+};
+MapsCache& maps_cache() {
+    static MapsCache c;
+    return c;
+}
+
 template <int CG, int U>
-cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+cudaError_t encode_maps(const Problem& p, const Tensors& t, EncodeTiledFn enc, bool x_direct, Maps* Mp,
+                        std::string* err) {
     using C = KCfg<CG, U>;
-    EncodeTiledFn enc = get_encode_fn(err);
-    if (!enc) return cudaErrorNotSupported;
-    Maps M;
+    Maps& M = *Mp;
     const int slices = p.D * p.naxes;
     const int Bp = p.MB * p.BM;
     if (!encode_blocked(enc, &M.x, t.xb, (long long)p.L0 * (p.H / 64) * Bp, err)) return cudaErrorInvalidValue;
@@ -947,8 +985,6 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     // away and the strided loads are off the dependency chain (x has no producer).  Same-box
     // C3 5.44 -> 5.40 ms, C4 0.922 -> 0.903 ms (profiles/r2_ab_x_direct.txt).  Grid inputs are
     // still packed.  FT_X_DIRECT=0 restores the pack (A/B).
-    const char* exd = getenv("FT_X_DIRECT");
-    const bool x_direct = p.kind == KIND_SEQ && (t.xsig != nullptr || !(exd && exd[0] == '0'));
     M.xd = M.x;
     if (x_direct) {
         const cuuint64_t dims[3] = {(cuuint64_t)p.H, (cuuint64_t)p.L0, (cuuint64_t)p.B};
@@ -988,16 +1024,15 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
             return cudaErrorInvalidValue;
     }
 
-    int dev = 0, nsm = 0;
-    cudaError_t e = cudaGetDevice(&dev);
-    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    if (e == cudaSuccess)
-        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
-    if (e != cudaSuccess) {
-        if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
-        return e;
-    }
+    return cudaSuccess;
+}
+
+template <int CG, int U>
+cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err,
+                           const Maps& M, bool x_direct, int dev, int nsm, int* clusters) {
+    using C = KCfg<CG, U>;
+    cudaError_t e = cudaSuccess;
+    const int Bp = p.MB * p.BM;
     // layer-0 inputs → blocked layout (part of the forward; ~T*H*Bp*4 bytes of traffic)
     {
         const long long nvec = (long long)p.L0 * (p.H / 64) * Bp * 8;
@@ -1036,11 +1071,14 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         cfg.gridDim = dim3((unsigned)(nsm & ~1));
         cfg.attrs = attr;
         cfg.numAttrs = 1;
-        int nclusters = 0;
-        e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U>, &cfg);
-        if (e != cudaSuccess || nclusters < 1) {
-            if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
-            return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
+        int nclusters = clusters[dev];
+        if (nclusters < 1) {
+            e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U>, &cfg);
+            if (e != cudaSuccess || nclusters < 1) {
+                if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
+                return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
+            }
+            clusters[dev] = nclusters;
         }
         grid = 2ll * nclusters;
         if (grid > 2 * p.ntiles) grid = 2 * p.ntiles;
@@ -1067,7 +1105,9 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
             p.naxes == 1 && p.D >= 2 && p.dil[0] == 1 && 2ll * p.NT <= grid / CG)
             q.owner = 2;
     }
-    if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // experiments
+#ifdef FT_DEV_EXPERIMENTS
+    if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // L2 policy experiments (dev builds)
+#endif
     if (q.band > 0) {
         q.resident_layers = p.D;  // every band's weights EVICT_LAST: resident while the band runs
         bool unit_dil = true;
@@ -1077,6 +1117,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         if (const char* e = getenv("FT_SKEW")) q.skew = atoi(e);
     }
     cudaLaunchAttribute attr2[2];
+    int nattr = 1;
     if (q.band == 0 && p.resident_layers == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM &&
         p.persist_layers != 0) {
         int maxp = 0, maxw = 0;
@@ -1104,6 +1145,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
             attr2[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
             cfg.attrs = attr2;
             cfg.numAttrs = 2;
+            nattr = 2;
         }
     }
     if (t.ysig_per_step) {  // every epilogue warp of every tile of a top-layer cell signals once
@@ -1111,9 +1153,51 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
                                ? q.naxes * q.MB * q.NT * CG * EPI_WARPS : 0;
         if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner == 1;  // owner walk: once per chunk
     }
-    e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
+    if constexpr (CG == 2)
+        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, wavefront_bf16_kernel<CG, U>, q, t, M);
+    else
+        e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
+}
+
+template <int CG, int U>
+cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+    using C = KCfg<CG, U>;
+    EncodeTiledFn enc = get_encode_fn(err);
+    if (!enc) return cudaErrorNotSupported;
+    int dev = 0, nsm = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess || dev < 0 || dev >= 64) {
+        if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
+        return e != cudaSuccess ? e : cudaErrorInvalidDevice;
+    }
+    const char* exd = getenv("FT_X_DIRECT");
+    const bool x_direct = p.kind == KIND_SEQ && (t.xsig != nullptr || !(exd && exd[0] == '0'));
+    MapsKey key;
+    std::memset(&key, 0, sizeof(key));
+    key = MapsKey{t.x, t.ys, t.W, t.U, t.hb, t.xb, t.yb, p.kind, p.cell, p.B, p.L0, p.L1, p.H, p.D,
+                  p.MB, p.BM, (int)x_direct, CG, U, dev};
+    Maps M;
+    if (!maps_cache().find(key, &M)) {
+        const cudaError_t ee = encode_maps<CG, U>(p, t, enc, x_direct, &M, err);
+        if (ee != cudaSuccess) return ee;
+        maps_cache().put(key, M);
+    }
+    // per-device one-time setup: the shared-memory opt-in and the cluster occupancy
+    static bool attr_set[64] = {};
+    static int clusters[64] = {};
+    if (!attr_set[dev]) {
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 C::SMEM_BYTES);
+        if (e != cudaSuccess) {
+            if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
+            return e;
+        }
+        attr_set[dev] = true;
+    }
+    return launch_cg_maps<CG, U>(p, t, s, err, M, x_direct, dev, nsm, clusters);
 }
 
 }  // namespace

@@ -471,9 +471,7 @@ cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStr
     attr[0].val.clusterDim.x = H / KU;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
-    cfg.attrs = attr;
-    cfg.numAttrs = 1;
-    e = cudaLaunchKernelEx(&cfg, wavefront_cluster_kernel, p, t, M);
+    e = launch_cluster_persistent(cfg, attr, 1, wavefront_cluster_kernel, p, t, M);
     if (e != cudaSuccess && err) *err = std::string("cluster launch: ") + cudaGetErrorString(e);
     return e;
 }

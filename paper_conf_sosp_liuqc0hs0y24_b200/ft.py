@@ -35,7 +35,11 @@ EXPORTS = (
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells", "ft_wavefront_cells_banded", "ft_tile_walk",
     "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
+    "ft_comm_unique_id", "ft_comm_init_rank", "ft_comm_gather_rank",
+    "ft_ipc_export", "ft_ipc_open", "ft_ipc_close",
 )
+FT_COMM_ID_BYTES = 128
+FT_IPC_HANDLE_BYTES = 64
 
 
 class FTError(RuntimeError):
@@ -93,6 +97,18 @@ def lib():
         L.ft_comm_gather.argtypes = [_c_vp, _c_vp, _c_vp, _c_vp, _c_int, _c_vp]
         L.ft_comm_destroy.restype = _c_int
         L.ft_comm_destroy.argtypes = [_c_vp]
+        L.ft_comm_unique_id.restype = _c_int
+        L.ft_comm_unique_id.argtypes = [_c_vp]
+        L.ft_comm_init_rank.restype = _c_int
+        L.ft_comm_init_rank.argtypes = [_c_int, _c_int, _c_vp, _c_int, ctypes.POINTER(_c_vp)]
+        L.ft_comm_gather_rank.restype = _c_int
+        L.ft_comm_gather_rank.argtypes = [_c_vp, _c_vp, _c_vp, _c_vp, _c_int, _c_vp]
+        L.ft_ipc_export.restype = _c_int
+        L.ft_ipc_export.argtypes = [_c_vp, _c_vp, ctypes.POINTER(_c_size)]
+        L.ft_ipc_open.restype = _c_int
+        L.ft_ipc_open.argtypes = [_c_vp, _c_size, _c_int, ctypes.POINTER(_c_vp)]
+        L.ft_ipc_close.restype = _c_int
+        L.ft_ipc_close.argtypes = [_c_vp, _c_size]
         L.ft_wavefront_cells.restype = _c_ll
         L.ft_wavefront_cells.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         L.ft_wavefront_cells_banded.restype = _c_ll
@@ -246,6 +262,46 @@ def ft_comm_gather(comm, send_ptrs, recv_ptr, nbytes, root, stream_ptrs):
 
 def ft_comm_destroy(comm):
     return lib().ft_comm_destroy(comm)
+
+
+def ft_comm_unique_id():
+    """Returns (status, bytes) — the opaque FT_COMM_ID_BYTES id one rank ships to the others."""
+    buf = ctypes.create_string_buffer(FT_COMM_ID_BYTES)
+    st = lib().ft_comm_unique_id(ctypes.cast(buf, _c_vp))
+    return st, buf.raw
+
+
+def ft_comm_init_rank(nranks, rank, uid, device):
+    """Returns (status, comm handle) — this process's rank of an NCCL communicator."""
+    buf = ctypes.create_string_buffer(bytes(uid), FT_COMM_ID_BYTES)
+    out = _c_vp()
+    st = lib().ft_comm_init_rank(nranks, rank, ctypes.cast(buf, _c_vp), device, ctypes.byref(out))
+    return st, out.value
+
+
+def ft_comm_gather_rank(comm, send_ptr, recv_ptr, nbytes, root, stream_ptr):
+    sizes = (_c_size * len(nbytes))(*nbytes)
+    return lib().ft_comm_gather_rank(comm, send_ptr, recv_ptr, ctypes.cast(sizes, _c_vp), root, stream_ptr)
+
+
+def ft_ipc_export(dev_ptr):
+    """Returns (status, handle bytes, offset) of the allocation holding `dev_ptr`."""
+    buf = ctypes.create_string_buffer(FT_IPC_HANDLE_BYTES)
+    off = _c_size()
+    st = lib().ft_ipc_export(dev_ptr, ctypes.cast(buf, _c_vp), ctypes.byref(off))
+    return st, buf.raw, off.value
+
+
+def ft_ipc_open(handle, offset, device):
+    """Returns (status, device pointer) of an exported allocation mapped into `device`."""
+    buf = ctypes.create_string_buffer(bytes(handle), FT_IPC_HANDLE_BYTES)
+    out = _c_vp()
+    st = lib().ft_ipc_open(ctypes.cast(buf, _c_vp), offset, device, ctypes.byref(out))
+    return st, out.value
+
+
+def ft_ipc_close(dev_ptr, offset):
+    return lib().ft_ipc_close(dev_ptr, offset)
 
 
 def check(status: int):

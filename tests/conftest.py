@@ -19,3 +19,22 @@ def cuda_device():
     if not torch.cuda.is_available():
         pytest.fail("GPU test selected but no CUDA device is visible")
     return torch.device("cuda:0")
+
+
+def pytest_sessionfinish(session, exitstatus):
+    """Dump the achieved parity errors the GPU tests recorded (tests/parity_log.py)."""
+    try:
+        from tests import parity_log
+    except ImportError:
+        try:
+            import parity_log
+        except ImportError:
+            return
+    if not parity_log.RECORDS:
+        return
+    import json
+    out = os.path.join(ROOT, "gpurun_out")
+    os.makedirs(out, exist_ok=True)
+    with open(os.path.join(out, "parity_errors.jsonl"), "w") as f:
+        for r in parity_log.RECORDS:
+            f.write(json.dumps(r) + "\n")

@@ -45,7 +45,8 @@ def test_set_l2_persist_validates():
     assert ft.ft_set_l2_persist(-2) == ft.FT_ERR_INVALID_ARGUMENT
     assert ft.ft_set_l2_persist(0) == ft.FT_OK
     assert ft.ft_set_l2_persist(32) == ft.FT_OK
-    assert ft.ft_set_l2_persist(-1) == ft.FT_OK  # back to the default
+    assert ft.ft_set_l2_persist(-1) == ft.FT_OK
+    assert ft.ft_set_l2_persist(0) == ft.FT_OK  # back to the default (off)
 
 
 FAKE = 1 << 20  # a 16-byte-aligned non-NULL "device" pointer; never dereferenced on error paths
@@ -128,6 +129,27 @@ def test_comm_validation():
     if not torch.cuda.is_available():
         st, comm = ft.ft_comm_create([0])
         assert st == ft.FT_ERR_CUDA and comm is None
+
+
+def test_comm_rank_and_ipc_validation():
+    """One-process-per-GPU gather and the peer-memory calls of the fused gather: argument checks
+    before any NCCL / CUDA work, and the two communicator forms refuse each other's gather."""
+    L = ft.lib()
+    assert L.ft_comm_unique_id(None) == ft.FT_ERR_INVALID_ARGUMENT
+    assert L.ft_comm_init_rank(2, 0, b"\0" * 128, 0, None) == ft.FT_ERR_INVALID_ARGUMENT
+    for nr, r in ((0, 0), (2, 2), (2, -1)):
+        st, comm = ft.ft_comm_init_rank(nr, r, b"\0" * 128, 0)
+        assert st == ft.FT_ERR_INVALID_ARGUMENT and comm is None
+    assert ft.ft_comm_gather_rank(None, FAKE, FAKE, [16, 16], 0, None) == ft.FT_ERR_INVALID_ARGUMENT
+    assert L.ft_ipc_export(None, None, None) == ft.FT_ERR_INVALID_ARGUMENT
+    assert L.ft_ipc_open(None, 0, 0, None) == ft.FT_ERR_INVALID_ARGUMENT
+    assert ft.ft_ipc_close(None, 0) == ft.FT_OK
+    import torch
+    if not torch.cuda.is_available():
+        st, comm = ft.ft_comm_init_rank(2, 0, b"\0" * 128, 0)
+        assert st == ft.FT_ERR_CUDA and comm is None
+        st, h, off = ft.ft_ipc_export(FAKE)
+        assert st != ft.FT_OK
 
 
 def test_valid_call_without_gpu_reports_cuda_error():

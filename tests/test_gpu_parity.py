@@ -14,6 +14,11 @@ import ftgen
 import oracle
 from paper_conf_sosp_liuqc0hs0y24_b200 import build, ft
 
+try:
+    from tests import parity_log
+except ImportError:
+    import parity_log
+
 pytestmark = pytest.mark.gpu
 
 F32_TOL = 1e-4
@@ -44,20 +49,32 @@ def normrel(a, ref):
     return maxabs(a, ref) / max(den, 1e-30)
 
 
+def rmsrel(a, ref):
+    den = float(np.sqrt(np.sum(ref * ref)))
+    return float(np.sqrt(np.sum((a - ref) ** 2))) / max(den, 1e-30)
+
+
 def _check(got, ref, dtype, keys, rows=None, ctx=""):
+    """Compare and record the achieved error (tests/parity_log.py); returns {key: (normwise,
+    rms-relative)}."""
+    errs = {}
     for k in keys:
-        g = host(got[k])
-        if rows is not None:
-            g = g[rows]
+        t = got[k]
+        if rows is not None:  # select the sampled rows on the device (h_all / c_all are GBs)
+            t = t[torch.as_tensor(rows, device=t.device)]
+        g = host(t)
         r = ref[k]
         assert g.shape == r.shape, (k, g.shape, r.shape)
         assert np.all(np.isfinite(g)), f"{ctx} {k}: non-finite output"
+        nw, rr, ma = normrel(g, r), rmsrel(g, r), maxabs(g, r)
+        parity_log.record(ctx, k, "f32" if dtype == torch.float32 else "bf16", nw, rr, ma,
+                          F32_TOL if dtype == torch.float32 else BF16_TOL)
+        errs[k] = (nw, rr)
         if dtype == torch.float32:
-            err = maxabs(g, r)
-            assert err <= F32_TOL, f"{ctx} {k}: max abs err {err:.3e} > {F32_TOL}"
+            assert ma <= F32_TOL, f"{ctx} {k}: max abs err {ma:.3e} > {F32_TOL}"
         else:
-            err = normrel(g, r)
-            assert err <= BF16_TOL, f"{ctx} {k}: normwise rel err {err:.3e} > {BF16_TOL}"
+            assert nw <= BF16_TOL, f"{ctx} {k}: normwise rel err {nw:.3e} > {BF16_TOL}"
+    return errs
 
 
 def _run_stacked(p, dtype, dil=None, want_all=False):
@@ -164,11 +181,47 @@ def test_bf16_cluster_stress_and_repeat(monkeypatch):
     _check(a, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="cluster repeat")
 
 
+def _record_bf16emu(p, rows, ref, ctx, dil=None):
+    """The precision floor: the oracle's bf16-emulating build (h rounded to bf16 after every
+    cell, the GPU's rounding point R20) against fp64 on the same rows — what a kernel with exact
+    fp32 arithmetic would achieve.  Recorded beside the GPU's error (diagnostic, never judged)."""
+    x = p["x"] if rows is None else p["x"][rows]
+    if dil is None:
+        emu = oracle.stacked_lstm(x, p["W"], p["U"], p["b"], precision="bf16emu", want_all=True)
+    else:
+        emu = oracle.dilated_rnn(x, p["W"], p["U"], p["b"], dil, precision="bf16emu", want_all=True)
+    return _record_emu(emu, ref, ctx)
+
+
+def _record_emu(emu, ref, ctx):
+    out = {}
+    for k in ref:
+        e = np.asarray(emu[k], dtype=np.float64)
+        out[k] = (normrel(e, ref[k]), rmsrel(e, ref[k]))
+        parity_log.record(ctx + " bf16emu-vs-f64", k, "bf16emu", out[k][0], out[k][1],
+                          maxabs(e, ref[k]), None)
+    return out
+
+
+def _assert_at_precision_floor(errs, emu, ctx):
+    """Regression bound well inside the 2e-2 tolerance: the GPU's error may exceed the exact-
+    rounding floor (bf16emu) only by what its fp32 reassociation and tanh.approx activations
+    add.  Measured (gpurun_out/parity_errors.jsonl): normwise within 1.2x of the
+    floor, RMS equal to it to 3 digits.  A 1.5x normwise / 1.1x RMS regression fails here,
+    and so does any normwise error above 5e-3."""
+    for k, (nw, rr) in errs.items():
+        fnw, frr = emu[k]
+        assert nw <= min(5e-3, 1.5 * fnw + 5e-4), f"{ctx} {k}: normwise {nw:.3e} vs floor {fnw:.3e}"
+        assert rr <= 1.1 * frr + 1e-4, f"{ctx} {k}: rms {rr:.3e} vs floor {frr:.3e}"
+
+
 def test_bf16_C2_full():
     c = ftgen.CONFIGS["C2"]
     p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C2"), "bf16")
     got = _run_stacked(p, torch.bfloat16, want_all=True)
-    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx="C2")
+    ref = _oracle_stacked(p, want_all=True)
+    errs = _check(got, ref, torch.bfloat16, ALL, ctx="C2")
+    _assert_at_precision_floor(errs, _record_bf16emu(p, None, ref, "C2"), "C2")
 
 
 def test_bf16_signal_preserving_scale():
@@ -208,10 +261,11 @@ def test_bf16_deterministic():
 def test_bf16_C3_sampled_rows():
     c = ftgen.CONFIGS["C3"]
     p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C3"), "bf16")
-    got = _run_stacked(p, torch.bfloat16)
-    rows = ftgen.sample_rows(c["batch"], 0, 1)[:4]
-    ref = _oracle_stacked(p, rows=rows)
-    _check(got, ref, torch.bfloat16, OUT, rows=rows, ctx="C3")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    rows = ftgen.sample_rows(c["batch"], 4, 1)  # SURVEY c.7: {0, 1, B/2, B-1} + 4 seeded rows
+    ref = _oracle_stacked(p, want_all=True, rows=rows)
+    errs = _check(got, ref, torch.bfloat16, ALL, rows=rows, ctx="C3")
+    _assert_at_precision_floor(errs, _record_bf16emu(p, rows, ref, "C3"), "C3")
 
 
 @pytest.mark.slow
@@ -219,9 +273,10 @@ def test_bf16_C4_sampled_rows():
     c = ftgen.CONFIGS["C4"]
     p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C4"), "bf16")
     got = _run_stacked(p, torch.bfloat16, dil=list(c["dilations"]))
-    rows = ftgen.sample_rows(c["batch"], 2, 2)
-    ref = _oracle_stacked(p, dil=list(c["dilations"]), rows=rows)
-    _check(got, ref, torch.bfloat16, OUT, rows=rows, ctx="C4")
+    rows = ftgen.sample_rows(c["batch"], 4, 2)
+    ref = _oracle_stacked(p, dil=list(c["dilations"]), rows=rows, want_all=True)
+    errs = _check(got, ref, torch.bfloat16, OUT, rows=rows, ctx="C4")
+    _assert_at_precision_floor(errs, _record_bf16emu(p, rows, ref, "C4", dil=list(c["dilations"])), "C4")
 
 
 @pytest.mark.slow
@@ -232,9 +287,11 @@ def test_bf16_C5_sampled_rows():
     args = [dev(g[k], torch.bfloat16) for k in ("x", "ys", "W", "U")] + [dev(g["b"], torch.float32)]
     got = ft.grid_rnn(*args)
     torch.cuda.synchronize()
-    rows = ftgen.sample_rows(c["batch"], 0, 3)[:4]
+    rows = ftgen.sample_rows(c["batch"], 4, 3)  # SURVEY c.7: {0, 1, B/2, B-1} + 4 seeded rows
     ref = oracle.grid_rnn(g["x"][rows], g["ys"][rows], g["W"], g["U"], g["b"])
-    _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n"), rows=rows, ctx="C5")
+    errs = _check(got, ref, torch.bfloat16, ("out", "h_n", "c_n"), rows=rows, ctx="C5")
+    emu = oracle.grid_rnn(g["x"][rows], g["ys"][rows], g["W"], g["U"], g["b"], precision="bf16emu")
+    _assert_at_precision_floor(errs, _record_emu(emu, ref, "C5"), "C5")
 
 
 # ------------------------------------------------------------------------- Listing 1 (NEXT-3)
@@ -326,10 +383,10 @@ def test_bf16_workspace_reuse_and_stream():
 # ------------------------------------------------------------------------- robustness
 @pytest.mark.parametrize("B,T,H,D,dil", [(130, 6, 128, 3, None), (256, 5, 64, 4, [1, 2, 3, 1])])
 def test_bf16_stress_delayed_release(B, T, H, D, dil, monkeypatch):
-    """Stress mode (FT_DEBUG=64): a pseudo-random delay before every counter release reorders
+    """Stress mode (FT_STRESS=1): a pseudo-random delay before every counter release reorders
     completions across CTAs; results must not change (shakes out missing acquire/release or
     proxy fences — SURVEY T6)."""
-    monkeypatch.setenv("FT_DEBUG", "64")
+    monkeypatch.setenv("FT_STRESS", "1")
     monkeypatch.setenv("FT_RESIDENT", "0")
     p = ftgen.stacked_inputs(B, T, H, D, 1717 + B, "bf16")
     got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
@@ -467,7 +524,7 @@ def test_bf16_l2_persist_window_bitwise_and_parity():
         assert ft.ft_set_l2_persist(8) == ft.FT_OK  # one layer
         one = _run_stacked(p, torch.bfloat16, want_all=True)
     finally:
-        ft.ft_set_l2_persist(-1)
+        ft.ft_set_l2_persist(0)  # back to the default (off)
     for k in ALL:  # the window changes where bytes come from, never the arithmetic
         assert torch.equal(off[k], on[k]), k
         assert torch.equal(off[k], one[k]), k
@@ -536,7 +593,7 @@ def test_bf16_layer_bands_stress(monkeypatch):
     monkeypatch.setenv("FT_BAND", "2")
     p = ftgen.stacked_inputs(256, 6, 128, 5, 1818, "bf16")
     first = _run_stacked(p, torch.bfloat16, want_all=True)
-    monkeypatch.setenv("FT_DEBUG", "64")
+    monkeypatch.setenv("FT_STRESS", "1")
     for _ in range(2):
         again = _run_stacked(p, torch.bfloat16, want_all=True)
         for k in ALL:
@@ -624,3 +681,59 @@ def test_c_abi_example_runs(tmp_path):
     assert r.returncode == 0, r.stdout + r.stderr
     assert "status OK, finite 1" in r.stdout, r.stdout
     assert "FT_ERR_UNSUPPORTED" in r.stdout, r.stdout
+
+
+# ------------------------------------------------------------------------- release hygiene
+def test_bf16_concurrent_streams_c3_class():
+    """Two C3-class forwards (CTA-pair cluster kernel, layer bands, owner walk) issued back to back
+    on two streams: each persistent launch needs every SM, so the library orders its launches
+    on a device one after another (PersistentOrder) instead of letting them split the SMs and
+    spin.  Both results match the oracle rows and a lone run bitwise."""
+    B, T, H, D = 256, 12, 1024, 8
+    pa = ftgen.stacked_inputs(B, T, H, D, 2121, "bf16")
+    pb = ftgen.stacked_inputs(B, T, H, D, 2122, "bf16")
+    args = {}
+    for name, p in (("a", pa), ("b", pb)):
+        args[name] = [dev(p[k], torch.bfloat16) for k in ("x", "W", "U")] + [dev(p["b"], torch.float32)]
+    alone = {n: ft.stacked_lstm(*args[n]) for n in ("a", "b")}
+    torch.cuda.synchronize()
+    sa, sb = torch.cuda.Stream(), torch.cuda.Stream()
+    wsa, wsb = ft.Workspace(), ft.Workspace()
+    for _ in range(3):
+        ra = ft.stacked_lstm(*args["a"], stream=sa, workspace=wsa)
+        rb = ft.stacked_lstm(*args["b"], stream=sb, workspace=wsb)
+    torch.cuda.synchronize()
+    for n, r in (("a", ra), ("b", rb)):
+        for k in OUT:
+            assert torch.equal(r[k], alone[n][k]), (n, k)
+    rows = [0, 255]
+    for n, p, r in (("a", pa, ra), ("b", pb, rb)):
+        _check(r, _oracle_stacked(p, rows=rows), torch.bfloat16, OUT, rows=rows, ctx=f"concurrent {n}")
+
+
+def test_bf16_concurrent_streams_cluster_kernel():
+    """The same for the DSMEM cluster kernel (C2 class) and the SMEM-resident kernel."""
+    p = ftgen.stacked_inputs(64, 16, 256, 4, 2123, "bf16")
+    a = [dev(p[k], torch.bfloat16) for k in ("x", "W", "U")] + [dev(p["b"], torch.float32)]
+    alone = ft.stacked_lstm(*a)
+    torch.cuda.synchronize()
+    ss = [torch.cuda.Stream() for _ in range(3)]
+    outs = [ft.stacked_lstm(*a, stream=s) for s in ss]
+    torch.cuda.synchronize()
+    for r in outs:
+        for k in OUT:
+            assert torch.equal(r[k], alone[k]), k
+
+
+def test_ft_debug_env_is_inert_in_release_build(monkeypatch):
+    """FT_DEBUG (result-invalidating timing experiments) exists only in development builds
+    (-DFT_DEV_EXPERIMENTS); setting it for the release libft.so changes nothing."""
+    p = ftgen.stacked_inputs(256, 9, 256, 3, 2124, "bf16")
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    base = _run_stacked(p, torch.bfloat16, want_all=True)
+    for bits in ("1", "2", "4", "16", "32", "255"):
+        monkeypatch.setenv("FT_DEBUG", bits)
+        got = _run_stacked(p, torch.bfloat16, want_all=True)
+        for k in ALL:
+            assert torch.equal(got[k], base[k]), (bits, k)
+    monkeypatch.delenv("FT_DEBUG")

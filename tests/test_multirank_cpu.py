@@ -59,3 +59,23 @@ def test_two_rank_batch_shard_gather_equals_single(tmp_path, B):
     ref = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"])
     for k in ("y", "h_n", "c_n"):
         assert np.array_equal(got[k], ref[k]), k
+
+
+def test_bench_refuses_to_mislabel_gpu_count():
+    """`bench.py --gpus N` never reports fewer ranks than asked: without N visible GPUs it exits 2
+    before printing a JSON line; under a torchrun whose WORLD_SIZE differs it exits 2 too."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    if torch.cuda.is_available():
+        pytest.skip("checks the no-device refusal")
+    env = dict(os.environ)
+    env.pop("FT_BENCH_SHARED_GPU", None)
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "2",
+                        "--warmup", "3"], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 2 and "needs 2 visible CUDA devices" in r.stderr
+    assert not [l for l in r.stdout.splitlines() if l.startswith("{")]
+    env.update(WORLD_SIZE="3", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "2",
+                        "--warmup", "3"], env=env, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 2 and "WORLD_SIZE=3 != --gpus 2" in r.stderr

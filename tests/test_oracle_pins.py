@@ -476,3 +476,21 @@ def test_bf16emu_within_precision_headroom():
         assert 0 < err < 5e-3, (k, err)
     bits = emu["h_all"].view(np.uint32)
     assert np.all((bits & 0xFFFF) == 0)
+
+
+# ------------------------------------------------------------------ CPU-baseline build (d.5)
+@pytest.mark.parametrize("precision", ["f64", "f32"])
+def test_timing_build_is_bitwise_the_parity_build(precision):
+    """bench.py's CPU baseline times the oracle built -O3 -march=native.
+    Same source, -ffp-contract=off, no -ffast-math: every output must be bitwise the parity
+    build's (C1, and a wider case that exercises the vectorised inner loops)."""
+    c = ftgen.CONFIGS["C1"]
+    cases = [ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], ftgen.config_seed("C1"),
+                                  "f32"),
+             ftgen.stacked_inputs(5, 6, 72, 3, 777, "bf16")]
+    for p in cases:
+        a = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision=precision, want_all=True)
+        b = oracle.stacked_lstm(p["x"], p["W"], p["U"], p["b"], precision=precision, want_all=True,
+                                build_kind="timing")
+        for k in a:
+            assert np.array_equal(a[k], b[k]), k
