@@ -19,6 +19,7 @@
 namespace {
 
 thread_local std::string g_last_error = "no error";
+thread_local std::string g_last_launch = "none";
 
 ft_status fail(ft_status s, const std::string& msg) {
     g_last_error = msg;
@@ -274,6 +275,7 @@ namespace ft {
 static int g_l2_persist_mib = 0;  // ft_set_l2_persist: 0 off (default), -1 auto, else MiB
 int l2_persist_mib() { return g_l2_persist_mib; }
 void set_last_error(const std::string& msg) { g_last_error = msg; }
+void set_last_launch(const std::string& s) { g_last_launch = s; }
 long long c_ring_elems(const Problem& p) {
     if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * c_slot_elems(p);
     return ((long long)p.D * 2 * p.L1 + (long long)p.D * p.L0 * 2) * c_slot_elems(p);
@@ -281,6 +283,8 @@ long long c_ring_elems(const Problem& p) {
 }  // namespace ft
 
 FT_API int ft_version(void) { return FT_VERSION; }
+
+FT_API const char* ft_last_launch(void) { return g_last_launch.c_str(); }
 
 FT_API ft_status ft_set_l2_persist(int mib) {
     if (mib < -1) return fail(FT_ERR_INVALID_ARGUMENT, "ft_set_l2_persist: mib must be >= -1");

@@ -57,9 +57,12 @@ struct Tensors {
 // cluster dimension (remembered per kernel), so the launch fails up front instead of spinning if
 // the grid cannot be co-resident.  Launches of the library on one device are additionally
 // ordered one after another (ft_api.cu PersistentOrder).
+// Text of the last forward launch on this thread (ft_last_launch): kernel, grid and schedule.
+void set_last_launch(const std::string& s);
+
 template <typename... KArgs, typename... Args>
 cudaError_t launch_cluster_persistent(cudaLaunchConfig_t cfg, const cudaLaunchAttribute* base, int nbase,
-                                      void (*kernel)(KArgs...), Args&&... args) {
+                                      int* cooperative, void (*kernel)(KArgs...), Args&&... args) {
     static int mode = 0;  // 0 untried, 1 cooperative + cluster accepted, 2 rejected
     cudaLaunchAttribute a[4];
     for (int i = 0; i < nbase && i < 3; ++i) a[i] = base[i];
@@ -71,6 +74,7 @@ cudaError_t launch_cluster_persistent(cudaLaunchConfig_t cfg, const cudaLaunchAt
         const cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
         if (e == cudaSuccess || mode == 1 || e == cudaErrorCooperativeLaunchTooLarge) {
             if (e == cudaSuccess) mode = 1;
+            if (cooperative) *cooperative = 1;
             return e;
         }
         cudaGetLastError();  // the combination is not supported here: plain cluster launch
@@ -78,6 +82,7 @@ cudaError_t launch_cluster_persistent(cudaLaunchConfig_t cfg, const cudaLaunchAt
     }
     cfg.attrs = a;
     cfg.numAttrs = nbase;
+    if (cooperative) *cooperative = 0;
     return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 

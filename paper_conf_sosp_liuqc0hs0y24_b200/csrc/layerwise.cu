@@ -542,6 +542,8 @@ cudaError_t launch_layerwise(int B, int T, int H, int D, const void* x, const vo
             if (err) *err = std::string("layerwise launch: ") + cudaGetErrorString(e);
             return e;
         }
+        set_last_launch("layerwise: per layer cuBLAS input GEMM + layer_recurrent_kernel grid=" +
+                        std::to_string(MB * NTR) + " cooperative=1 (x" + std::to_string(D) + " layers)");
         X = a.out;
     }
     return cudaSuccess;

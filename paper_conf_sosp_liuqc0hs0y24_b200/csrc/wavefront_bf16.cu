@@ -1153,10 +1153,20 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
                                ? q.naxes * q.MB * q.NT * CG * EPI_WARPS : 0;
         if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner == 1;  // owner walk: once per chunk
     }
+    int coop = 1;
     if constexpr (CG == 2)
-        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, wavefront_bf16_kernel<CG, U>, q, t, M);
+        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, &coop, wavefront_bf16_kernel<CG, U>,
+                                      q, t, M);
     else
         e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
+    if (e == cudaSuccess)
+        set_last_launch("wavefront_bf16_kernel<" + std::to_string(CG) + "," + std::to_string(U) +
+                        "> grid=" + std::to_string(grid) + " cluster=" + std::to_string(CG) +
+                        " cooperative=" + std::to_string(coop) + " band=" + std::to_string(q.band) +
+                        " skew=" + std::to_string(seq_skew(q)) + " owner=" + std::to_string(q.owner) +
+                        " x_direct=" + std::to_string(q.x_direct) + " persist_layers=" +
+                        std::to_string(q.persist_layers) + " resident_layers=" +
+                        std::to_string(q.resident_layers) + " stress=" + std::to_string((q.debug & 64) != 0));
     if (e != cudaSuccess && err) *err = std::string("bf16 launch: ") + cudaGetErrorString(e);
     return e;
 }

@@ -471,7 +471,11 @@ cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStr
     attr[0].val.clusterDim.x = H / KU;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
-    e = launch_cluster_persistent(cfg, attr, 1, wavefront_cluster_kernel, p, t, M);
+    int coop = 0;
+    e = launch_cluster_persistent(cfg, attr, 1, &coop, wavefront_cluster_kernel, p, t, M);
+    if (e == cudaSuccess)
+        set_last_launch("wavefront_cluster_kernel grid=" + std::to_string(p.D * (H / KU)) + " cluster=" +
+                        std::to_string(H / KU) + " cooperative=" + std::to_string(coop));
     if (e != cudaSuccess && err) *err = std::string("cluster launch: ") + cudaGetErrorString(e);
     return e;
 }

@@ -175,6 +175,7 @@ cudaError_t launch_wavefront_f32(const Problem& p, const Tensors& t, cudaStream_
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     e = cudaLaunchKernelEx(&cfg, wavefront_f32_kernel, p, t);
+    if (e == cudaSuccess) set_last_launch("wavefront_f32_kernel grid=" + std::to_string(grid) + " cooperative=1");
     if (e != cudaSuccess && err) *err = std::string("f32 launch: ") + cudaGetErrorString(e);
     return e;
 }

@@ -363,6 +363,9 @@ cudaError_t launch_resident_t(const Problem& p, const Tensors& t, cudaStream_t s
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     e = cudaLaunchKernelEx(&cfg, wavefront_resident_kernel<BNUR>, p, t, M);
+    if (e == cudaSuccess)
+        set_last_launch("wavefront_resident_kernel<" + std::to_string(BNUR) + "> grid=" +
+                        std::to_string(p.D * (H / BNUR)) + " cooperative=1");
     if (e != cudaSuccess && err) *err = std::string("resident launch: ") + cudaGetErrorString(e);
     return e;
 }

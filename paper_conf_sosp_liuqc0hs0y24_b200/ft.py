@@ -25,7 +25,7 @@ FT_MAX_DEPTH = 64
 
 # every symbol include/ft.h declares (checked by tests/test_abi.py against the header)
 EXPORTS = (
-    "ft_version", "ft_status_string", "ft_last_error", "ft_set_l2_persist",
+    "ft_version", "ft_status_string", "ft_last_error", "ft_last_launch", "ft_set_l2_persist",
     "ft_stacked_lstm_workspace_size", "ft_stacked_lstm_fwd",
     "ft_stacked_lstm_hostio_workspace_size", "ft_stacked_lstm_fwd_hostio",
     "ft_stacked_rnn_workspace_size", "ft_stacked_rnn_fwd",
@@ -65,6 +65,7 @@ def lib():
         L.ft_status_string.restype = ctypes.c_char_p
         L.ft_status_string.argtypes = [_c_int]
         L.ft_last_error.restype = ctypes.c_char_p
+        L.ft_last_launch.restype = ctypes.c_char_p
         L.ft_stacked_lstm_workspace_size.restype = _c_size
         L.ft_stacked_lstm_workspace_size.argtypes = [_c_int] * 6
         L.ft_dilated_rnn_workspace_size.restype = _c_size
@@ -135,6 +136,11 @@ def status_string(s: int) -> str:
 
 def ft_last_error() -> str:
     return lib().ft_last_error().decode()
+
+
+def ft_last_launch() -> str:
+    """Launch configuration and schedule of the last forward on this thread (diagnostic)."""
+    return lib().ft_last_launch().decode()
 
 
 def ft_stacked_lstm_workspace_size(batch, seq, hidden, depth, dt, h_all_provided):
