@@ -90,10 +90,6 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
     p->NT = (H + p->BNU - 1) / p->BNU;
     p->ncells = (long long)D * L0 * L1;
     p->ntiles = p->ncells * p->naxes * p->MB * p->NT;
-    // bf16: TMA row coordinates into the blocked buffers are int32
-    if (dt == FT_BF16 && (ft::hb_rows_total(*p) >= (1ll << 31) ||
-                          (long long)L0 * (H / 64) * p->MB * p->BM >= (1ll << 31)))
-        return fail(FT_ERR_UNSUPPORTED, "problem too large: blocked activation rows exceed int32 TMA coordinates");
     if (kind == ft::KIND_SEQ) {
         int off = 0;
         for (int d = 0; d < D; ++d) {
@@ -103,7 +99,23 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
             off += (int)len;
         }
         p->ring_off[D] = off;
+        // a6 for the bf16 streaming kernel: the SSA buffer hb as per-layer rings (ft_common.cuh
+        // hb_slot_row) plus two T-step regions for band-boundary layers — C3: 1600 rows of
+        // (d, t) → 16·4 + 200.  The launcher lays the slots out once the band is known.
+        if (dt == FT_BF16 && cell == ft::CELL_LSTM && ft::hb_ring_eligible(*p)) {
+            long long rows = 2ll * L0;
+            for (int d = 0; d < D; ++d) rows += ft::hb_ring_len(dil[d], L0);
+            if (rows < (long long)D * L0) {
+                p->hring = 1;
+                p->hb_rows = (int)rows;
+                ft::hb_layout(*p, 0);  // the paper order's layout; the launcher redoes it per band
+            }
+        }
     }
+    // bf16: TMA row coordinates into the blocked buffers are int32
+    if (dt == FT_BF16 && (ft::hb_rows_total(*p) >= (1ll << 31) ||
+                          (long long)L0 * (H / 64) * p->MB * p->BM >= (1ll << 31)))
+        return fail(FT_ERR_UNSUPPORTED, "problem too large: blocked activation rows exceed int32 TMA coordinates");
     return FT_OK;
 }
 
@@ -124,7 +136,7 @@ WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
     w.hall_off = w.ring_off + w.ring_bytes;
-    if (dt == FT_BF16)  // the blocked SSA activation buffer (always; the caller's h_all is a copy)
+    if (dt == FT_BF16)  // the blocked SSA activation buffer (full, or per-layer rings: p.hring)
         w.hall_bytes = round_up((size_t)ft::hb_rows_total(p) * 64 * 2, 256);
     else
         w.hall_bytes = h_all_provided
@@ -779,4 +791,26 @@ FT_API ft_status ft_b2b_gemm_fwd(int M, int N, int K, int P, ft_dtype dt, const 
     cudaError_t e = ft::launch_b2b_gemm(M, N, A, B, C, D, static_cast<cudaStream_t>(stream), &err);
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, err.empty() ? cudaGetErrorString(e) : err);
     return FT_OK;
+}
+
+FT_API long long ft_ssa_slots(int depth, int seq, const int* dilations, int band, int* off, int* mask) {
+    if (depth <= 0 || seq <= 0 || depth > FT_MAX_DEPTH || !dilations || !off || !mask) return -1;
+    ft::Problem p;
+    std::memset(&p, 0, sizeof(p));
+    p.kind = ft::KIND_SEQ;
+    p.D = depth;
+    p.L0 = seq;
+    p.L1 = 1;
+    long long rows = 2ll * seq;
+    for (int d = 0; d < depth; ++d) {
+        if (dilations[d] < 1) return -1;
+        p.dil[d] = dilations[d];
+        rows += ft::hb_ring_len(dilations[d], seq);
+    }
+    ft::hb_layout(p, band > 0 && band < depth ? band : 0);
+    for (int d = 0; d < depth; ++d) {
+        off[d] = p.hb_off[d];
+        mask[d] = p.hb_mask[d];
+    }
+    return rows;
 }

@@ -63,6 +63,11 @@ struct Problem {
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
+    int hring;           // bf16 streaming KIND_SEQ: hb holds a ring of slots per layer instead of
+                         // every (d, t) row (see hb_slot_row); 0 = one row per (d, t)
+    int hb_rows;         // hring: rows of hb the workspace reserves (Σ ring lengths + 2·L0)
+    int hb_off[FT_MAX_DEPTH];   // hring: first hb row of layer d's slots
+    int hb_mask[FT_MAX_DEPTH];  // hring: slot of step t = t & hb_mask[d] (-1: one slot per step)
     long long ncells;    // D*L0*L1
     long long ntiles;    // ncells * naxes * MB * NT
     int dil[FT_MAX_DEPTH];           // KIND_SEQ: per-layer dilation (1 = stacked)
@@ -428,6 +433,48 @@ FT_HD int h_rows(const Problem& p) {
 FT_HD int h_row(const Problem& p, int d, int i, int j, int a) {
     return p.kind == KIND_SEQ ? d * p.L0 + i : ((d * p.L0 + i) * p.L1 + j) * 2 + a;
 }
+// Row of the blocked SSA buffer hb that holds h(d, i, j, axis).  Without a ring it is the
+// logical row h_row().  With p.hring (bf16 streaming stacked / dilated nests) layer d owns
+// slots [hb_off[d], hb_off[d] + len) and step t lives in slot t & hb_mask[d]: the SSA node of
+// §4.4 (L217) needs each h only until its consumers have read it — (d, t + s_d) through the
+// recurrence and (d + 1, t) through the depth edge (Table 4).  The writer of a wrapped slot waits
+// for the depth consumer of the slot's previous step (run_epilogue); the recurrent consumer is
+// an ancestor of the writer when len is a multiple of 2·s_d.  A band's last layer (read by the
+// next band, which runs after it) keeps every step (hb_mask = -1) in one of two alternating
+// regions.
+FT_HD int hb_slot_row(const Problem& p, int d, int i, int j, int a) {
+    if (p.kind == KIND_SEQ && p.hring) return p.hb_off[d] + (i & p.hb_mask[d]);
+    return h_row(p, d, i, j, a);
+}
+// Ring length of a stacked / dilated layer: the smallest power of two >= max(4, 2·s) when s is a
+// power of two (then a multiple of 2·s, see hb_slot_row), else no wrap; never more than T.
+FT_HD int hb_ring_len(int s, int T) {
+    if (s & (s - 1)) return T;
+    int r = 4;
+    while (r < 2 * s) r <<= 1;
+    return r < T ? r : T;
+}
+
+// Slot layout of the hb rings for layer bands of width `band` (0 = one band, the paper order):
+// layer d gets hb_ring_len(s_d, T) slots at a running offset; a band's last layer (except the
+// last band's) instead keeps all T steps in region (band index & 1) after the rings — the next
+// band reads it after this band is done, and the band after that writes the same region only
+// after the next band's first layer has read it (a chain of depth edges orders them).
+inline void hb_layout(Problem& p, int band) {
+    int off = 0;
+    for (int d = 0; d < p.D; ++d) {
+        const int len = hb_ring_len(p.dil[d], p.L0);
+        p.hb_off[d] = off;
+        p.hb_mask[d] = len < p.L0 ? len - 1 : -1;
+        off += len;
+    }
+    if (band > 0 && band < p.D)
+        for (int d = band - 1; d < p.D - 1; d += band) {
+            p.hb_off[d] = off + ((d / band) & 1) * p.L0;
+            p.hb_mask[d] = -1;
+        }
+}
+
 // K rows of one U slice: H (seq) or 2H (grid, acting on s = [h^x; h^y]).
 FT_HD int u_krows(const Problem& p) { return p.kind == KIND_SEQ ? p.H : 2 * p.H; }
 
@@ -440,11 +487,11 @@ FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
     const Cell& c = tl.cell;
     if (p.kind == KIND_SEQ) {
         seg[0] = (c.d == 0) ? Segment{SRC_X, c.i, W_IN, 0, 0, -1, 0}
-                            : Segment{SRC_H, h_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0,
+                            : Segment{SRC_H, hb_slot_row(p, c.d - 1, c.i, 0, 0), W_IN, c.d, 0,
                                       (int)cell_lin(p, c.d - 1, c.i, 0), 0};
         const int s = p.dil[c.d];
         const bool rec = c.i >= s && p.cell == CELL_LSTM;  // the linear cell has no h@U term
-        seg[1] = Segment{rec ? SRC_H : SRC_NONE, rec ? h_row(p, c.d, c.i - s, 0, 0) : 0,
+        seg[1] = Segment{rec ? SRC_H : SRC_NONE, rec ? hb_slot_row(p, c.d, c.i - s, 0, 0) : 0,
                          W_REC, c.d, 0, rec ? (int)cell_lin(p, c.d, c.i - s, 0) : -1, 0};
         seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0, -1, 0};
     } else {
@@ -524,7 +571,8 @@ FT_HD long long c_producer(const Problem& p, const TileId& tl, int* pi, int* pj)
 // so that the A operand of one tile K-chunk (128 batch rows x 64 units) is one contiguous 16 KiB
 // block: a 2-D TMA box with no large strides, and the epilogue's h stores are coalesced.
 FT_HD long long hb_rows_total(const Problem& p) {
-    return (long long)h_rows(p) * (p.H / 64) * ((long long)p.MB * p.BM);
+    return (long long)(p.kind == KIND_SEQ && p.hring ? p.hb_rows : h_rows(p)) * (p.H / 64) *
+           ((long long)p.MB * p.BM);
 }
 FT_HD long long hb_row(const Problem& p, int row, int kc, int b) {
     return ((long long)row * (p.H / 64) + kc) * ((long long)p.MB * p.BM) + b;

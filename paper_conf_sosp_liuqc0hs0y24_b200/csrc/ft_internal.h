@@ -104,6 +104,10 @@ int bf16_kernel_choice(const Problem& p);
 // NEXT-4 back-to-back GEMMs (b2b_gemm.cu): D[M][64] = (A[M][64] @ B[64][N]) @ C[N][64]
 cudaError_t launch_b2b_gemm(int M, int N, const void* A, const void* B, const void* C, float* D,
                             cudaStream_t s, std::string* err);
+// a6: whether a bf16 stacked / dilated LSTM keeps hb as per-layer rings (p.hring): every problem
+// the streaming kernel runs — i.e. not one of the small SMEM-resident / DSMEM-cluster shapes,
+// which keep one hb row per (d, t)
+bool hb_ring_eligible(const Problem& p);
 // a5 weight-resident mode (wavefront_resident.cu): slab width 16/32 when the weights fit, else 0
 int resident_bnu(const Problem& p, int nsm);
 bool cluster_kernel_applies(const Problem& p);

@@ -537,6 +537,15 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         FT_TR_BEGIN();
         if (cprod >= 0 && leader_thread && !own && !FT_DEV_BIT(P.debug, 1))
             wait_flag_geq(T.flags + (split ? cflag_index(P, cprod, tl.m) : cprod * P.MB + tl.m), target);
+        // hb ring (p.hring): this tile's h goes to the slot of step t − len, whose depth consumer
+        // (d + 1, t − len) must have read it (its counter completes after its MMAs consumed the
+        // operands).  An earlier tile of the wavefront / owner order, so waiting cannot deadlock;
+        // it is normally long done (the wait sits before the accumulator wait, off the chain).
+        if (P.hring && leader_thread && c.d + 1 < P.D) {
+            const int mask = P.hb_mask[c.d];
+            if (mask >= 0 && c.i > mask)
+                wait_flag_geq(T.flags + cell_lin(P, c.d + 1, c.i - mask - 1, 0) * P.MB + tl.m, target);
+        }
         named_bar_sync(1, EPI_THREADS);
         if (leader_thread) FT_TR_END(TR_E_CFLAG);
         // cst: the previous c on entry, updated in place to this tile's c' by the math loop
@@ -572,7 +581,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         const uint32_t tbase = tmem_base + (uint32_t)(acc * C::BN) + ((uint32_t)(q * 32) << 16) +
                                (uint32_t)(half * EPI_UNITS);
         uint4 hp[EPI_UNITS / 8];
-        const int row_h = h_row(P, c.d, c.i, c.j, tl.axis);
+        const int row_h = hb_slot_row(P, c.d, c.i, c.j, tl.axis);
 #pragma unroll
         for (int u0 = 0; u0 < EPI_UNITS; u0 += CH) {
             __syncwarp();  // tcgen05.ld is .sync.aligned: the whole warp, converged
@@ -1096,6 +1105,7 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
     q.flag_mult = CG * EPI_WARPS;  // every epilogue warp of every CTA of a tile releases once
     q.x_direct = x_direct;
     q.band = choose_band(p, (int)(grid / CG));
+    if (q.hring) hb_layout(q, q.band);
     // Dedicated owners for layer 0 of a dilated nest (TileWalk owner mode 2: layer 0 has
     // dilation 1, the only recurrence without slack) measured slower on C4 (0.916-0.920 ->
     // 0.958 ms, profiles/r2_ab_layer0_owner.txt): the chain is not queueing behind other
@@ -1232,7 +1242,15 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned l
 }
 #endif
 
+bool hb_ring_eligible(const Problem& p) {
+    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM) return false;
+    if (p.B <= ROWS && resident_bnu(p, 148) != 0) return false;  // SMEM-resident candidate
+    if (p.B <= 64 && (p.H == 128 || p.H == 256)) return false;    // DSMEM-cluster candidate
+    return true;
+}
+
 int bf16_kernel_choice(const Problem& p) {
+    if (p.hring) return 2;  // laid out for the streaming kernel (hb_ring_eligible)
     // latency-bound small stacked LSTMs (C2): weights resident in the SMEM of one cluster per
     // layer, h exchanged through DSMEM on the time edge (wavefront_cluster.cu)
     const char* envc = getenv("FT_CLUSTER");  // "0" disables it (comparisons)

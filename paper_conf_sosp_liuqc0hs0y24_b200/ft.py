@@ -33,7 +33,7 @@ EXPORTS = (
     "ft_b2b_gemm_fwd",
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
-    "ft_wavefront_cells", "ft_wavefront_cells_banded", "ft_tile_walk",
+    "ft_wavefront_cells", "ft_wavefront_cells_banded", "ft_tile_walk", "ft_ssa_slots",
     "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
     "ft_comm_unique_id", "ft_comm_init_rank", "ft_comm_gather_rank",
     "ft_ipc_export", "ft_ipc_open", "ft_ipc_close",
@@ -115,6 +115,8 @@ def lib():
         L.ft_wavefront_cells_banded.restype = _c_ll
         L.ft_wavefront_cells_banded.argtypes = [_c_int] * 6 + [_c_vp, _c_ll]
         L.ft_tile_walk.restype = _c_ll
+        L.ft_ssa_slots.restype = _c_ll
+        L.ft_ssa_slots.argtypes = [_c_int, _c_int, _c_vp, _c_int, _c_vp, _c_vp]
         L.ft_tile_walk.argtypes = [_c_int] * 8 + [_c_vp, _c_ll]
         _lib = L
     return _lib
@@ -247,6 +249,18 @@ def ft_tile_walk(depth, seq, band, skew, owner, ntiles_n, worker, nworkers):
     buf = (ctypes.c_int * (3 * max(n, 1)))()
     lib().ft_tile_walk(depth, seq, band, skew, owner, ntiles_n, worker, nworkers, ctypes.cast(buf, _c_vp), n)
     return [tuple(buf[3 * k:3 * k + 3]) for k in range(n)]
+
+
+def ft_ssa_slots(depth, seq, dilations, band):
+    """(rows, off[], mask[]) of the streaming kernel's SSA ring layout — host only."""
+    dil = _int_array(dilations)
+    off = (ctypes.c_int * depth)()
+    mask = (ctypes.c_int * depth)()
+    rows = lib().ft_ssa_slots(depth, seq, ctypes.cast(dil, _c_vp), band, ctypes.cast(off, _c_vp),
+                              ctypes.cast(mask, _c_vp))
+    if rows < 0:
+        raise FTError(FT_ERR_INVALID_ARGUMENT, "bad ssa-slot query")
+    return rows, list(off), list(mask)
 
 
 def ft_comm_create(devices):

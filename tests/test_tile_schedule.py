@@ -292,3 +292,66 @@ def test_grid_depth_bands_are_legal(D, Lx, Ly, band):
     bands = [c[1] // band for c in cells]
     assert bands == sorted(bands)
     assert ft.ft_wavefront_cells_banded(1, D, Lx, Ly, D, 1) == ft.ft_wavefront_cells(1, D, Lx, Ly)
+
+
+# ------------------------------------------------------------------ SSA slot rings (a6)
+def _simulate_ssa_rings(D, T, dil, band, seed):
+    """Random legal executions of the nest against the kernel's hb slot layout (ft_ssa_slots).
+    Events: start(d,t) reads h(d-1,t) and h(d,t-s) from their slots (needs both producers
+    ended); end(d,t) writes h(d,t) into its slot, and — as run_epilogue does — waits first for
+    the depth consumer (d+1, t-len) of the slot's previous step when the slot wraps.  Every read
+    must find the step it expects; every event order the dependences allow is possible, so this
+    covers the banded owner walk and the round-robin wavefront alike."""
+    import random
+    rows, off, mask = ft.ft_ssa_slots(D, T, dil, band)
+    rng = random.Random(seed)
+    slot = {}
+    started, ended = set(), set()
+
+    def row(d, t):
+        r = off[d] + (t & mask[d])
+        assert 0 <= r < rows
+        return r
+
+    def can_start(d, t):
+        return ((d == 0 or (d - 1, t) in ended) and (t < dil[d] or (d, t - dil[d]) in ended))
+
+    def can_end(d, t):
+        if (d, t) not in started:
+            return False
+        m = mask[d]
+        if m >= 0 and t > m and d + 1 < D:
+            return (d + 1, t - m - 1) in ended
+        return True
+
+    cells = [(d, t) for d in range(D) for t in range(T)]
+    while len(ended) < len(cells):
+        enabled = [("s", c) for c in cells if c not in started and can_start(*c)]
+        enabled += [("e", c) for c in cells if c in started and c not in ended and can_end(*c)]
+        assert enabled, "deadlock: the back-pressure wait blocked every cell"
+        kind, (d, t) = rng.choice(enabled)
+        if kind == "s":
+            if d > 0:
+                assert slot.get(row(d - 1, t)) == (d - 1, t), ("depth read", d, t)
+            if t >= dil[d]:
+                assert slot.get(row(d, t - dil[d])) == (d, t - dil[d]), ("recurrent read", d, t)
+            started.add((d, t))
+        else:
+            slot[row(d, t)] = (d, t)
+            ended.add((d, t))
+
+
+@pytest.mark.parametrize("D,T,dil,band", [
+    (6, 17, [1] * 6, 0), (8, 13, [1] * 8, 4), (8, 13, [1] * 8, 3), (5, 21, [1] * 5, 2),
+    (6, 40, [1, 2, 4, 8, 16, 32], 0), (4, 19, [3, 1, 7, 2], 0), (7, 9, [1] * 7, 2)])
+def test_ssa_ring_layout_is_safe_under_every_order(D, T, dil, band):
+    for seed in range(6):
+        _simulate_ssa_rings(D, T, dil, band, seed)
+
+
+def test_ssa_ring_layout_sizes():
+    rows, off, mask = ft.ft_ssa_slots(16, 100, [1] * 16, 4)  # C3: 16·4 ring slots + 2·T
+    assert rows == 16 * 4 + 200
+    assert [m for m in mask].count(-1) == 3  # the boundary layers of bands 0..2
+    rows, off, mask = ft.ft_ssa_slots(6, 100, [1, 2, 4, 8, 16, 32], 0)  # C4
+    assert mask == [3, 3, 7, 15, 31, 63]
