@@ -52,35 +52,19 @@ struct Tensors {
                                    // last step of the chunk), so a chunk completes at per_step
 };
 
-// Persistent cluster launch: a cluster grid sized by cudaOccupancyMaxActiveClusters fits the idle
-// device, and the cooperative attribute is added as well when the driver accepts it next to the
-// cluster dimension (remembered per kernel), so the launch fails up front instead of spinning if
-// the grid cannot be co-resident.  Launches of the library on one device are additionally
-// ordered one after another (ft_api.cu PersistentOrder).
 // Text of the last forward launch on this thread (ft_last_launch): kernel, grid and schedule.
 void set_last_launch(const std::string& s);
 
+// Persistent cluster launch.  The cluster grid is sized by cudaOccupancyMaxActiveClusters, so on
+// an otherwise idle device every CTA is resident at once.  (The cooperative attribute next to the
+// cluster dimension was tried: the driver accepts it, but Nsight Compute's kernel replay then
+// fails with LaunchFailed, so it is not used.)  Launches of this library on one device are
+// ordered one after another (ft_api.cu PersistentOrder), so two of its persistent kernels never
+// split the SMs; another application's kernel can only delay CTAs until it finishes.
 template <typename... KArgs, typename... Args>
 cudaError_t launch_cluster_persistent(cudaLaunchConfig_t cfg, const cudaLaunchAttribute* base, int nbase,
                                       int* cooperative, void (*kernel)(KArgs...), Args&&... args) {
-    static int mode = 0;  // 0 untried, 1 cooperative + cluster accepted, 2 rejected
-    cudaLaunchAttribute a[4];
-    for (int i = 0; i < nbase && i < 3; ++i) a[i] = base[i];
-    if (mode != 2) {
-        a[nbase].id = cudaLaunchAttributeCooperative;
-        a[nbase].val.cooperative = 1;
-        cfg.attrs = a;
-        cfg.numAttrs = nbase + 1;
-        const cudaError_t e = cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
-        if (e == cudaSuccess || mode == 1 || e == cudaErrorCooperativeLaunchTooLarge) {
-            if (e == cudaSuccess) mode = 1;
-            if (cooperative) *cooperative = 1;
-            return e;
-        }
-        cudaGetLastError();  // the combination is not supported here: plain cluster launch
-        mode = 2;
-    }
-    cfg.attrs = a;
+    cfg.attrs = const_cast<cudaLaunchAttribute*>(base);
     cfg.numAttrs = nbase;
     if (cooperative) *cooperative = 0;
     return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
