@@ -64,9 +64,12 @@ enum TraceSlot {
 __device__ unsigned long long g_trace[1024 * TR_SLOTS];
 // per-tile event timestamps (%globaltimer, ns) of the leader CTA: 0 wait start, 1 deps ready,
 // 2 A loads issued, 3 MMA done (epilogue saw tfull), 4 counter released, 5 last producer flag
-// acquired, 6 MMA warp got the accumulator, 7 MMA warp issued the last chunk
-constexpr int EV_MAX_TILES = 65536;
-constexpr int EV_K = 8;
+// acquired, 6 MMA warp got the accumulator, 7 MMA warp issued the last chunk, 8 A producer got
+// the slot of the last segment's first chunk, 9 A producer got the slot of the tile's last
+// chunk, 10 MMA saw the last segment's first chunk land, 11 MMA saw the chunk before it land,
+// 12 weight producer issued the tile's last weight chunk
+constexpr int EV_MAX_TILES = 32768;
+constexpr int EV_K = 16;
 __device__ unsigned long long g_events[EV_MAX_TILES * EV_K];
 #define FT_EV(tile, k) do { if ((tile) < EV_MAX_TILES) g_events[(tile) * EV_K + (k)] = globaltimer_ns(); } while (0)
 // register accumulators, flushed once per role (keeps the instrumented loops lean)
@@ -267,6 +270,12 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             if constexpr (kWeights) FT_TR_BEGIN();
             mbar_wait(&empty[stage], phase ^ 1);
             if constexpr (kWeights) FT_TR_END(TR_P_EMPTY);
+#ifdef FT_TRACE
+            if constexpr (!kWeights) {
+                if (rank == 0 && c == nchunks - kchunks) FT_EV(tile, 8);
+                if (rank == 0 && c == nchunks - 1) FT_EV(tile, 9);
+            }
+#endif
             const uint32_t bar = full0 + 8u * (uint32_t)stage;
             if (rank == 0) mbar_arrive_expect_tx(&full[stage], tx);
             if constexpr (kWeights) {
@@ -289,6 +298,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             }
         }
         if constexpr (!kWeights) if (rank == 0) FT_EV(tile, 2);
+        if constexpr (kWeights) if (rank == 0) FT_EV(tile, 12);
     }
     FT_TR_FLUSH(true);  // the two producers fill disjoint slots
 }
@@ -327,6 +337,10 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
             FT_TR_BEGIN();
             mbar_wait_warp(&full[stage], phase);
             FT_TR_END(TR_M_FULL);
+#ifdef FT_TRACE
+            if ((threadIdx.x & 31) == 0 && c == nchunks - kchunks) FT_EV(tile, 10);
+            if ((threadIdx.x & 31) == 0 && c == nchunks - kchunks - 1) FT_EV(tile, 11);
+#endif
             tc_fence_after();
             if (elect_one()) {
                 if (FT_DEV_BIT(P.debug, 4)) {  // timing experiment: no MMA, hand the slot straight back

@@ -49,7 +49,7 @@ for l in sys.stdin:
                FT_LIB_PATH=build/ab/libft_$v.so QT_REPS=${QT_REPS:-30} timeout 600 python tools/quick_time.py ${cfgs//,/ } 2>&1 | sed "s/^/$v /" >> "$f"
              done; done; cat "$f";;
     dram:*)  rest=${step#dram:}; lib=${rest%%:*}; cf=${rest#*:}; f=$(out "dram_${lib}_${cf}")
-             FT_LIB_PATH=build/ab/libft_$lib.so QT_REPS=3 QT_WARM=2 timeout 900 ncu --metrics \
+             FT_LIB_PATH=build/ab/libft_$lib.so QT_REPS=3 QT_WARM=2 timeout 300 ncu --metrics \
                gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum,lts__t_bytes.sum,sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed \
                --clock-control none -k regex:wavefront -s 2 -c 1 --csv python tools/quick_time.py "$cf" > "$f" 2>&1
              grep -E "dram__|gpu__time|lts__t_bytes|tensor_cycles" "$f" | awk -F'","' '{print $(NF-2), $(NF-1), $NF}';;
