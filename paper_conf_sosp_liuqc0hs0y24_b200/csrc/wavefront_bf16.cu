@@ -1120,12 +1120,18 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
     q.x_direct = x_direct;
     q.band = choose_band(p, (int)(grid / CG));
     if (q.hring) hb_layout(q, q.band);
-    // Dedicated owners for layer 0 of a dilated nest (TileWalk owner mode 2: layer 0 has
-    // dilation 1, the only recurrence without slack) measured slower on C4 (0.916-0.920 ->
-    // 0.958 ms, profiles/r2_ab_layer0_owner.txt): the chain is not queueing behind other
-    // layers' tiles.  Opt-in only (FT_OWNER_L0=1).
-    if (const char* e = getenv("FT_OWNER_L0")) {
-        if (atoi(e) != 0 && q.band == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.MB == 1 &&
+    // Dedicated owners for layer 0 of a dilated nest (TileWalk owner mode 2): layer 0 has
+    // dilation 1, the only recurrence without slack, so its slabs get their own CTA pairs (cell
+    // state in registers, no queueing behind other layers' tiles); the other layers run
+    // round-robin on the rest.  Round 1 measured it slower (C4 0.916 -> 0.958 ms); with the
+    // round-2 epilogue and launch path it is faster: C4 0.838 -> 0.798 ms same-box
+    // (profiles/rnd2_ab_c4_owner_l0.txt).  Default for dilated nests; FT_OWNER_L0=0 turns it off.
+    {
+        bool dilated = false;
+        for (int d = 1; d < p.D; ++d) dilated = dilated || p.dil[d] > 1;
+        const char* e = getenv("FT_OWNER_L0");
+        const bool want = e ? atoi(e) != 0 : dilated;
+        if (want && q.band == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.MB == 1 &&
             p.naxes == 1 && p.D >= 2 && p.dil[0] == 1 && 2ll * p.NT <= grid / CG)
             q.owner = 2;
     }

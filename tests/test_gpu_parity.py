@@ -640,14 +640,17 @@ def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
 
 @pytest.mark.parametrize("dil", [[1, 2, 4, 8, 16, 32], [1, 3, 2]])
 def test_bf16_layer0_owner_walk(dil, monkeypatch):
-    """Opt-in layer-0 owners (TileWalk mode 2) for dilated nests: parity and bitwise equality
-    with the default round-robin walk."""
+    """Layer-0 owners (TileWalk mode 2, the default for dilated nests): parity and bitwise
+    equality with the round-robin walk (FT_OWNER_L0=0)."""
     monkeypatch.setenv("FT_RESIDENT", "0")
     D = len(dil)
     p = ftgen.stacked_inputs(256, 9, 128, D, 2020 + D, "bf16")
+    monkeypatch.setenv("FT_OWNER_L0", "0")
     ref_gpu = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
-    monkeypatch.setenv("FT_OWNER_L0", "1")
+    assert "owner=0" in ft.ft_last_launch()
+    monkeypatch.delenv("FT_OWNER_L0")
     got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    assert "owner=2" in ft.ft_last_launch()
     _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"l0 owner {dil}")
     for k in ALL:
         assert torch.equal(got[k], ref_gpu[k]), k
