@@ -361,7 +361,7 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
         tl.axis = 0;
         tl.m = 0;
         tl.n = w.n;
-        tid = cell_lin(p, 0, w.t, 0) * p.NT + w.n;
+        tid = p.ncells * p.NT + (long long)w.t * p.NT + w.n;  // (trace ids past the other tiles')
         ++w.t;
         return true;
     }

@@ -6,7 +6,9 @@ so the step time is the critical chain.  Per step (medians over t):
   land   E2     -> E7       loads landed + last MMA chunk issued
   tail   E7     -> E3       MMA completion seen by the epilogue
   epi    E3     -> E4       epilogue (TMEM -> math -> h stores -> release)
-usage: python tools/chain_anatomy.py B T H UNITS"""
+usage: python tools/chain_anatomy.py B T H UNITS [owner]
+  owner: a 2-layer dilated nest (dilations 1, T) whose layer 0 runs on the layer-0 owners;
+  the anatomy is layer 0's."""
 import ctypes
 import os
 import sys
@@ -19,23 +21,34 @@ import ftgen  # noqa: E402
 from paper_conf_sosp_liuqc0hs0y24_b200 import ft  # noqa: E402
 
 B, T, H, U = (int(v) for v in sys.argv[1:5])
+OWNER = len(sys.argv) > 5 and sys.argv[5] == "owner"
 os.environ["FT_TILE_UNITS"] = str(U)
 os.environ["FT_RESIDENT"] = "0"
 ft.LIB_PATH = os.path.abspath(os.environ.get("FT_TRACE_LIB", "build/trace/libft_trace.so"))
 L = ft.lib()
-p = ftgen.stacked_inputs(B, T, H, 1, 1, "bf16")
+p = ftgen.stacked_inputs(B, T, H, 2 if OWNER else 1, 1, "bf16")
 a = [torch.from_numpy(p[k]).cuda().to(torch.bfloat16) for k in ("x", "W", "U")] + [torch.from_numpy(p["b"]).cuda()]
 ws = ft.Workspace()
 for _ in range(4):
-    ft.stacked_lstm(*a, workspace=ws)
+    ft.stacked_lstm(*a, workspace=ws, dilations=[1, T] if OWNER else None)
 torch.cuda.synchronize()
+print(ft.ft_last_launch())
 NT = H // U
-n = T * NT
 EVK = 16
-buf = (ctypes.c_ulonglong * (n * EVK))()
-L.ft_debug_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
-L.ft_debug_events(buf, n)
-ev = np.array(buf[:], dtype=np.float64).reshape(T, NT, EVK)
+if OWNER:  # layer-0 owner tiles are traced at ids ncells*NT + t*NT0 + n
+    NT0 = NT
+    base = 2 * T * NT
+    n = base + T * NT0
+    buf = (ctypes.c_ulonglong * (n * EVK))()
+    L.ft_debug_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
+    L.ft_debug_events(buf, n)
+    ev = np.array(buf[:], dtype=np.float64)[base * EVK:].reshape(T, NT0, EVK)
+else:
+    n = T * NT
+    buf = (ctypes.c_ulonglong * (n * EVK))()
+    L.ft_debug_events.argtypes = [ctypes.c_void_p, ctypes.c_int]
+    L.ft_debug_events(buf, n)
+    ev = np.array(buf[:], dtype=np.float64).reshape(T, NT, EVK)
 ev = (ev - ev[ev > 0].min()) / 1000.0
 R = ev[:, :, 4].max(1)
 E5, E2, E7, E3 = (ev[:, :, k].max(1) for k in (5, 2, 7, 3))
