@@ -941,12 +941,17 @@ int choose_band(const Problem& p, int workers) {
     }
     if (p.kind == KIND_GRID) {
         // grid nests carry two fp32 cell states per cell (c^x, c^y); their rings for all depths
-        // are D · 2 · (Lx + Ly) slots of B·H fp32.  When that exceeds a 64 MiB L2 budget (C5:
-        // 128 MiB), run depth bands whose rings fit: C5 DRAM 9.6 -> 2.9 GB per forward (band 2),
-        // 6.30 -> 6.07 ms same-box (profiles/r2_ab_grid_bands.txt)
+        // are D · 2 · (Lx + Ly) slots of B·H fp32.  A depth band's live L2 set is its rings plus
+        // its weights (2 axes x 4 gates x H x 3H bf16 per depth); when the whole nest's set exceeds
+        // a 64 MiB L2 budget (C5: 128 MiB of rings + 48 MiB of weights), run depth bands whose set
+        // fits.  C5: band 1 (32 + 12 MiB).  Same box: DRAM 9.6 GB (paper order) -> 5.9 GB (bands
+        // of 2) -> 2.95 GB (bands of 1) per forward at the same time (5.94 / 5.95 ms,
+        // profiles/r2_ab_grid_bands.txt, profiles/rnd2_ab_c5_band1.txt)
         const double ring_per_depth = 2.0 * (p.L0 + p.L1) * (double)p.B * p.H * 4.0;
-        if (ring_per_depth * p.D <= 64.0 * 1024 * 1024) return 0;
-        const int band = (int)((64.0 * 1024 * 1024) / ring_per_depth);
+        const double w_per_depth = 2.0 * 4.0 * p.H * 3.0 * p.H * 2.0;
+        const double per_depth = ring_per_depth + w_per_depth;
+        if (per_depth * p.D <= 64.0 * 1024 * 1024) return 0;
+        const int band = (int)((64.0 * 1024 * 1024) / per_depth);
         return band < 1 ? 1 : (band >= p.D ? 0 : band);
     }
     if (p.kind != KIND_SEQ) return 0;
