@@ -34,7 +34,7 @@ def test_exports_every_header_symbol():
 
 
 def test_version_and_status_strings():
-    assert ft.ft_version() == 100
+    assert ft.ft_version() == 200
     assert ft.status_string(ft.FT_OK) == "FT_OK"
     assert ft.status_string(ft.FT_ERR_UNSUPPORTED) == "FT_ERR_UNSUPPORTED"
     assert ft.status_string(ft.FT_ERR_WORKSPACE_TOO_SMALL) == "FT_ERR_WORKSPACE_TOO_SMALL"
