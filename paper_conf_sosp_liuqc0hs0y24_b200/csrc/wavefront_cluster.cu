@@ -17,8 +17,8 @@
 //
 // Shapes: batch B <= 64 (the tile is M = 128 with rows >= B never stored), H in {128, 256}
 // (cluster of H/32 <= 8 CTAs), stacked (dilation 1).  N = 4 gates x 32 units = 128, K = 64 per
-// chunk.  Warps: 0 TMA producer, 1 MMA issuer (whole warp), 2–5 epilogue (warps of TMEM lane
-// quadrants 0 and 1, i.e. rows 0..63, do the work).
+// chunk.  Warps: 0 TMA producer, 1 MMA issuer (whole warp), 4, 5, 8, 9 epilogue (the warps of
+// TMEM lane quadrants 0 and 1, i.e. rows 0..63, two per quadrant with 16 units each).
 //
 // Recurrent operand layout (no swizzle, K-major): k-group g (8 units, 16 bytes) of all 64 rows is
 // one contiguous 1 KiB block (row r at r*16), so CTA j's 32 units = k-groups 4j..4j+3 = ONE
@@ -64,7 +64,14 @@ constexpr int KB = 64;      // batch rows actually carried (B <= KB)
 constexpr int KU = 32;      // hidden units per CTA
 constexpr int KN = 4 * KU;  // UMMA N (i | f | o | ĝ)
 constexpr int KBK = 64;     // K per chunk
-constexpr int KTHREADS = 192;
+// 10 warps: 0 TMA, 1 MMA, and the epilogue warps whose TMEM lane quadrant (warp % 4) holds the
+// batch rows 0..63 — warps 4, 5 (units 0..15 of the slice) and 8, 9 (units 16..31).  Warps 2, 3,
+// 6, 7 sit on quadrants 2, 3 (rows >= 64, never stored) and only join the final barriers.
+// (Round 1 had 6 warps with 2 working epilogue warps of 32 units each: the gate math of a step
+// then took ~1.0 us; split over 4 warps it halves, tools/latency_bench.cu.)
+constexpr int KTHREADS = 320;
+constexpr int KEPI = 4;                // working epilogue warps
+constexpr int KEU = KU / 2;            // units per epilogue thread
 constexpr int XSTAGES = 3;
 constexpr int X_BYTES = KB * KBK * 2;          // 8 KiB: 64 rows x 64 units (SW128)
 constexpr int GATE_BYTES = KU * KBK * 2;       // 4 KiB: one gate's 32 units x 64 K (SW64)
@@ -143,7 +150,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
         }
         for (int a = 0; a < 2; ++a) {
             mbar_init(&tfull[a], 1);
-            mbar_init(&tempty[a], 2);  // the two working epilogue warps
+            mbar_init(&tempty[a], KEPI);  // the working epilogue warps
             mbar_init(&hfull[a], 1);
         }
         mbar_init(wbar, 1);
@@ -153,7 +160,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
         mbar_arrive_expect_tx(&hfull[0], rec_bytes);
         mbar_arrive_expect_tx(&hfull[1], rec_bytes);
     }
-    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * KU) {
+    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * KU) {  // (4·KU = 128 <= 256 threads past warp 1)
         const int e = threadIdx.x - 64;
         sbias[e] = T.b[(long long)d * 4 * P.H + (e / KU) * P.H + (int)j * KU + e % KU];
     }
@@ -258,15 +265,16 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
             acc ^= 1;
             if (acc == 0) acc_phase ^= 1;
         }
-    } else if ((warp & 3) < 2) {
-        // ---- epilogue: warps of TMEM lane quadrants 0 and 1 (rows 0..63); c in registers ------
-        const int q = warp & 3, row = q * 32 + lane;
+    } else if (warp >= 4 && (warp & 3) < 2) {
+        // ---- epilogue: warps of TMEM lane quadrants 0 and 1 (rows 0..63), KEU units each; c in
+        //      registers.  half = which 16 units of the CTA's 32-unit slice this warp owns.
+        const int q = warp & 3, row = q * 32 + lane, half = warp >= 8;
         const bool valid = row < P.B;
-        const int n0 = (int)j * KU;
+        const int n0 = (int)j * KU + half * KEU;
         const bool sender = (warp == 4 && lane == 0);
-        float creg[KU];
+        float creg[KEU];
 #pragma unroll
-        for (int u = 0; u < KU; ++u) creg[u] = 0.f;
+        for (int u = 0; u < KEU; ++u) creg[u] = 0.f;
         __nv_bfloat16* hb = (__nv_bfloat16*)T.hb;
         __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
         int acc = 0;
@@ -275,58 +283,59 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
             mbar_wait(&tfull[acc], acc_phase);
             if (sender) FT_CEV(t, 2);
             tc_fence_after();
-            const uint32_t tbase = tmem_base + (uint32_t)(acc * KN) + ((uint32_t)(q * 32) << 16);
-            uint32_t hp[KU / 2];
-#pragma unroll
-            for (int u0 = 0; u0 < KU; u0 += 16) {
-                float zi[16], zf[16], zo[16], zg[16];
-                tmem_ld_32x32b_x16(tbase + 0 * KU + u0, zi);
-                tmem_ld_32x32b_x16(tbase + 1 * KU + u0, zf);
-                tmem_ld_32x32b_x16(tbase + 2 * KU + u0, zo);
-                tmem_ld_32x32b_x16(tbase + 3 * KU + u0, zg);
+            const uint32_t tbase = tmem_base + (uint32_t)(acc * KN) + ((uint32_t)(q * 32) << 16) + half * KEU;
+            uint32_t hp[KEU / 2];
+            {
+                float zi[KEU], zf[KEU], zo[KEU], zg[KEU];
+                tmem_ld_32x32b_x16(tbase + 0 * KU, zi);
+                tmem_ld_32x32b_x16(tbase + 1 * KU, zf);
+                tmem_ld_32x32b_x16(tbase + 2 * KU, zo);
+                tmem_ld_32x32b_x16(tbase + 3 * KU, zg);
                 tmem_wait_ld();
-                if (u0 + 16 == KU) {
-                    tc_fence_before();
-                    __syncwarp();
-                    if (lane == 0) mbar_arrive(&tempty[acc]);
-                }
+                tc_fence_before();
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&tempty[acc]);
+                const int ub = half * KEU;
+                // (1) the time edge first, pipelined with the math: as soon as a k-group of 8 units
+                //     is done, every thread st.async's its row of it (16 B) straight from registers
+                //     into every cluster CTA's buffer t & 1, each store carrying complete_tx(16) to
+                //     that CTA's hfull[t & 1] (no staging, no barrier); the next k-group's math
+                //     overlaps those stores in flight
+                const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES + (uint32_t)half * 2048u +
+                                           (uint32_t)row * 16u;
+                const uint32_t bar_local = smem_u32(&hfull[t & 1]);
 #pragma unroll
-                for (int v = 0; v < 16; ++v) {
-                    const float ig = sigmoid_approx(zi[v] + sbias[0 * KU + u0 + v]);
-                    const float fg = sigmoid_approx(zf[v] + sbias[1 * KU + u0 + v]);
-                    const float og = sigmoid_approx(zo[v] + sbias[2 * KU + u0 + v]);
-                    const float gh = tanh_approx(zg[v] + sbias[3 * KU + u0 + v]);
-                    creg[u0 + v] = fmaf(fg, creg[u0 + v], ig * gh);
-                    zi[v] = og * tanh_approx(creg[u0 + v]);  // h
+                for (int g = 0; g < KEU / 8; ++g) {
+#pragma unroll
+                    for (int v = 8 * g; v < 8 * g + 8; ++v) {
+                        const float ig = sigmoid_approx(zi[v] + sbias[0 * KU + ub + v]);
+                        const float fg = sigmoid_approx(zf[v] + sbias[1 * KU + ub + v]);
+                        const float og = sigmoid_approx(zo[v] + sbias[2 * KU + ub + v]);
+                        const float gh = tanh_approx(zg[v] + sbias[3 * KU + ub + v]);
+                        creg[v] = fmaf(fg, creg[v], ig * gh);
+                        zi[v] = og * tanh_approx(creg[v]);  // h
+                    }
+#pragma unroll
+                    for (int v = 4 * g; v < 4 * g + 4; ++v) hp[v] = kpack(zi[2 * v], zi[2 * v + 1]);
+                    if (t + 1 < P.L0) {
+                        const uint4 val = make_uint4(hp[4 * g], hp[4 * g + 1], hp[4 * g + 2], hp[4 * g + 3]);
+                        for (int r = 0; r < CS; ++r)
+                            st_async_v4(mapa_shared(dst_local, (uint32_t)r) + g * 1024u, val,
+                                        mapa_shared(bar_local, (uint32_t)r));
+                    }
                 }
                 if (sender) FT_CEV(t, 3);
-#pragma unroll
-                for (int v = 0; v < 8; ++v) hp[u0 / 2 + v] = kpack(zi[2 * v], zi[2 * v + 1]);
             }
-            // (1) the time edge first: every thread st.async's its row of the slice (4 x 16 B)
-            //     straight from registers into every cluster CTA's buffer t & 1, each store
-            //     carrying complete_tx(16) to that CTA's hfull[t & 1] (no staging, no barrier)
-            if (t + 1 < P.L0) {
-                const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES + (uint32_t)row * 16u;
-                const uint32_t bar_local = smem_u32(&hfull[t & 1]);
-                for (int r = 0; r < CS; ++r) {
-                    const uint32_t dst = mapa_shared(dst_local, (uint32_t)r);
-                    const uint32_t mb = mapa_shared(bar_local, (uint32_t)r);
-#pragma unroll
-                    for (int g = 0; g < KU / 8; ++g)
-                        st_async_v4(dst + g * 1024u, make_uint4(hp[4 * g], hp[4 * g + 1], hp[4 * g + 2], hp[4 * g + 3]), mb);
-                }
-                if (sender) FT_CEV(t, 4);
-            }
+            if (sender) FT_CEV(t, 4);
             // (2) the depth edge: h into the blocked SSA buffer, then one cumulative release
             const Cell cell{d + t, d, t, 0};
             if (valid) {
                 uint4* dst = reinterpret_cast<uint4*>(hb + hb_row(P, h_row(P, d, t, 0, 0), n0 / 64, row) * 64 + (n0 % 64));
 #pragma unroll
-                for (int w = 0; w < KU / 8; ++w)
+                for (int w = 0; w < KEU / 8; ++w)
                     __stcg(dst + w, make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]));
             }
-            named_bar_sync(1, 64);
+            named_bar_sync(1, KEPI * 32);
             if (sender && d + 1 < P.D) red_release_gpu_add(T.flags + cell_lin(P, d, t, 0), 1);
             // (3) outputs nobody inside the nest reads
             if (valid) {
@@ -334,30 +343,30 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
                 if (h_all) {
                     uint4* dh = reinterpret_cast<uint4*>(h_all + hi);
 #pragma unroll
-                    for (int w = 0; w < KU / 8; ++w)
+                    for (int w = 0; w < KEU / 8; ++w)
                         dh[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
                 }
                 if (T.c_all) {
                     float4* dc = reinterpret_cast<float4*>(T.c_all + hi);
 #pragma unroll
-                    for (int w = 0; w < KU / 4; ++w)
+                    for (int w = 0; w < KEU / 4; ++w)
                         dc[w] = make_float4(creg[4 * w], creg[4 * w + 1], creg[4 * w + 2], creg[4 * w + 3]);
                 }
                 if (d == P.D - 1) {
                     uint4* dy = reinterpret_cast<uint4*>((__nv_bfloat16*)T.y + y_index(P, cell, 0, row, n0));
 #pragma unroll
-                    for (int w = 0; w < KU / 8; ++w)
+                    for (int w = 0; w < KEU / 8; ++w)
                         dy[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
                 }
                 if (t == P.L0 - 1) {
                     const long long ni = hn_index(P, cell, 0, row, n0);
                     uint4* dn = reinterpret_cast<uint4*>((__nv_bfloat16*)T.h_n + ni);
 #pragma unroll
-                    for (int w = 0; w < KU / 8; ++w)
+                    for (int w = 0; w < KEU / 8; ++w)
                         dn[w] = make_uint4(hp[4 * w], hp[4 * w + 1], hp[4 * w + 2], hp[4 * w + 3]);
                     float4* dc = reinterpret_cast<float4*>(T.c_n + ni);
 #pragma unroll
-                    for (int w = 0; w < KU / 4; ++w)
+                    for (int w = 0; w < KEU / 4; ++w)
                         dc[w] = make_float4(creg[4 * w], creg[4 * w + 1], creg[4 * w + 2], creg[4 * w + 3]);
                 }
             }
