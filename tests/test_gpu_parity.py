@@ -740,3 +740,30 @@ def test_ft_debug_env_is_inert_in_release_build(monkeypatch):
         for k in ALL:
             assert torch.equal(got[k], base[k]), (bits, k)
     monkeypatch.delenv("FT_DEBUG")
+
+
+# ------------------------------------------------------------------------- SSA slot rings (a6)
+@pytest.mark.parametrize("B,T,H,D,dil,band", [
+    (256, 41, 128, 6, None, "2"),            # stacked, bands of 2: rings of 4 wrap 10x, boundary regions alternate
+    (256, 41, 128, 6, None, "0"),            # paper order: every layer a ring
+    (256, 40, 64, 5, [1, 2, 4, 8, 3], "0"),  # dilated: rings 4, 4, 8, 16 and a non-power-of-two layer (no wrap)
+    (130, 19, 64, 64, None, "8"),            # FT_MAX_DEPTH layers in bands of 8
+])
+def test_bf16_ssa_rings(B, T, H, D, dil, band, monkeypatch):
+    """The streaming kernel's SSA buffer is a ring of slots per layer (ft_common.cuh hb_slot_row):
+    long sequences wrap every ring many times, under bands and in the paper order.  Outputs,
+    including h_all / c_all written from registers, match the oracle on sampled rows and are
+    bitwise equal across schedules."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    monkeypatch.setenv("FT_BAND", band)
+    p = ftgen.stacked_inputs(B, T, H, D, 3131 + D, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    rows = ftgen.sample_rows(B, 2, 5)
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True, rows=rows), torch.bfloat16, ALL, rows=rows,
+           ctx=f"ssa ring {B, T, H, D, dil, band}")
+    rows_s, off, mask = ft.ft_ssa_slots(D, T, dil or [1] * D, int(band))
+    assert any(m >= 0 for m in mask)  # some layer really wraps
+    monkeypatch.setenv("FT_BAND", "0" if band != "0" else "3")
+    other = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    for k in ALL:
+        assert torch.equal(got[k], other[k]), k
