@@ -399,14 +399,23 @@ def run_ours(args):
             "c_n": torch.empty((B, D, H), dtype=torch.float32, device=dev)}
     from paper_conf_sosp_liuqc0hs0y24_b200.shard import CommGather, PeerGather
     gat = None
+    gather_fallback = None
     if gather == "fused":
         # NEXT-1: y / h_n / c_n stored by the kernel epilogue straight into rank 0's buffers
         # (peer memory mapped by the library's ft_ipc_* calls; NVLink on an NVSwitch node)
         gat = PeerGather(B * world, T, H, D, bf, dev, dst=0)
-        outs = gat.local()
-    elif gather == "nccl":
+        if not gat.ok():  # every rank agrees; fall back to the library's NCCL gather
+            gather_fallback = f"fused gather unavailable ({gat.error or 'on another rank'}); used nccl"
+            gat.close()
+            gat, gather = None, ("nccl" if not shared else "none")
+    if gather == "nccl":
         # the library's own NCCL gather (ft_comm_gather_rank), rank 0 in place
         gat = CommGather(B * world, T, H, D, bf, dev, dst=0)
+        if not gat.ok():
+            gather_fallback = (gather_fallback or "") + f"; nccl gather unavailable ({gat.error or 'on another rank'})"
+            gat.close()
+            gat, gather = None, "none"
+    if gat is not None:
         outs = gat.local()
     stream = torch.cuda.current_stream()
 
@@ -555,7 +564,7 @@ def run_ours(args):
         "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
         "data": "synthetic (ftgen splitmix64: x~U(-1,1), W,U,b~U(+-1/sqrt(H)), bf16 RNE)",
         "config": dict(workload_config(n_gpus), gather=gather,
-                       gather_note={"none": "no output gather (one rank)",
+                       gather_note={"none": "no output gather",
                                     "fused": "y/h_n/c_n stored by every rank's kernel epilogue into "
                                              "rank 0's buffers (peer memory, ft_ipc_*), inside the "
                                              "timed step",
@@ -564,6 +573,7 @@ def run_ours(args):
                        control_plane=backend if world > 1 else None,
                        ranks_share_one_gpu=bool(shared) if world > 1 else None),
         "gather_ok": gather_ok,
+        "gather_fallback": gather_fallback,
         "parity": parity,
         "tensor_pipe_pct_of_peak": 100.0 * roofline["frac"],
         "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,

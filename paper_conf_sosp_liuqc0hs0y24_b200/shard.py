@@ -91,23 +91,42 @@ class PeerGather:
         self.device = torch.device(device)
         self.shapes = _out_shapes(total_rows, seq, hidden, depth, dtype)
         self.full, self.opened = None, {}
+        self.error = None  # set when this rank could not export / map the buffers (no exception:
+                           # every rank still takes part in the collectives; see ok())
+        handles = None
         if self.rank == dst:
             self.full = {k: torch.empty(shp, dtype=dt, device=self.device) for k, (shp, dt) in self.shapes.items()}
             handles = {}
             for k, v in self.full.items():
                 st, h, off = ft.ft_ipc_export(v.data_ptr())
-                ft.check(st)
+                if st != ft.FT_OK:
+                    self.error = f"ft_ipc_export: {ft.ft_last_error()}"
+                    handles = {"error": self.error}
+                    break
                 handles[k] = (h, off)
-        else:
-            handles = None
         obj = [handles]
         dist.broadcast_object_list(obj, src=dst, group=group)
         if self.rank != dst:
-            dev = self.device.index if self.device.index is not None else torch.cuda.current_device()
-            for k, (h, off) in obj[0].items():
-                st, ptr = ft.ft_ipc_open(h, off, dev)
-                ft.check(st)
-                self.opened[k] = (ptr, off)
+            if "error" in obj[0]:
+                self.error = "root: " + obj[0]["error"]
+            else:
+                dev = self.device.index if self.device.index is not None else torch.cuda.current_device()
+                for k, (h, off) in obj[0].items():
+                    st, ptr = ft.ft_ipc_open(h, off, dev)
+                    if st != ft.FT_OK:
+                        self.error = f"ft_ipc_open: {ft.ft_last_error()}"
+                        break
+                    self.opened[k] = (ptr, off)
+
+    def ok(self):
+        """Collective: True when every rank mapped the buffers (else close() and fall back)."""
+        import torch
+        import torch.distributed as dist
+        t = torch.tensor([0 if self.error else 1], dtype=torch.int32)
+        if dist.get_backend(self.group) == "nccl":
+            t = t.cuda()
+        dist.all_reduce(t, op=dist.ReduceOp.MIN, group=self.group)
+        return bool(t.item())
 
     def local(self):
         """This rank's row slice of the destination buffers (pass as `out=` to stacked_lstm)."""
@@ -156,16 +175,23 @@ class CommGather:
         self.world = dist.get_world_size(group)
         self.total_rows = total_rows
         self.shapes = _out_shapes(total_rows, seq, hidden, depth, dtype)
+        self.error, self.comm = None, None
         uid = None
         if self.rank == 0:
             st, uid = ft.ft_comm_unique_id()
-            ft.check(st)
+            if st != ft.FT_OK:
+                uid = None
         obj = [uid]
         dist.broadcast_object_list(obj, src=0, group=group)
         dev = torch.device(device)
-        st, self.comm = ft.ft_comm_init_rank(self.world, self.rank, obj[0],
-                                             dev.index if dev.index is not None else torch.cuda.current_device())
-        ft.check(st)
+        if obj[0] is None:
+            self.error = "ft_comm_unique_id failed on rank 0"
+        else:
+            st, self.comm = ft.ft_comm_init_rank(self.world, self.rank, obj[0],
+                                                 dev.index if dev.index is not None else torch.cuda.current_device())
+            if st != ft.FT_OK:
+                self.error = f"ft_comm_init_rank: {ft.ft_last_error()}"
+                self.comm = None
         self.full = None
         if self.rank == dst:
             self.full = {k: torch.empty(shp, dtype=dt, device=dev) for k, (shp, dt) in self.shapes.items()}
@@ -187,6 +213,16 @@ class CommGather:
         dev = torch.device("cuda", torch.cuda.current_device())
         return {k: torch.empty((b - a,) + tuple(shp[1:]), dtype=dt, device=dev)
                 for k, (shp, dt) in self.shapes.items()}
+
+    def ok(self):
+        """Collective: True when every rank has a communicator."""
+        import torch
+        import torch.distributed as dist
+        t = torch.tensor([0 if self.error else 1], dtype=torch.int32)
+        if dist.get_backend() == "nccl":
+            t = t.cuda()
+        dist.all_reduce(t, op=dist.ReduceOp.MIN)
+        return bool(t.item())
 
     def gather(self, outs, stream_ptr):
         from . import ft
