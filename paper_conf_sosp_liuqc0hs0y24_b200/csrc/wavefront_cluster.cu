@@ -61,23 +61,31 @@ using namespace sm100;
 
 constexpr int KROWS = 128;  // UMMA M
 constexpr int KB = 64;      // batch rows actually carried (B <= KB)
-constexpr int KU = 32;      // hidden units per CTA
-constexpr int KN = 4 * KU;  // UMMA N (i | f | o | ĝ)
 constexpr int KBK = 64;     // K per chunk
 // 10 warps: 0 TMA, 1 MMA, and the epilogue warps whose TMEM lane quadrant (warp % 4) holds the
-// batch rows 0..63 — warps 4, 5 (units 0..15 of the slice) and 8, 9 (units 16..31).  Warps 2, 3,
-// 6, 7 sit on quadrants 2, 3 (rows >= 64, never stored) and only join the final barriers.
-// (Round 1 had 6 warps with 2 working epilogue warps of 32 units each: the gate math of a step
-// then took ~1.0 us; split over 4 warps it halves, tools/latency_bench.cu.)
+// batch rows 0..63 — warps 4, 5 (the first half of the CTA's units) and 8, 9 (the second half).
+// Warps 2, 3, 6, 7 sit on quadrants 2, 3 (rows >= 64, never stored) and only join the final
+// barriers.  (Round 1 had 6 warps with 2 working epilogue warps of 32 units each: the gate math
+// of a step then took ~1.0 us; split over 4 warps it halves, tools/latency_bench.cu.)
 constexpr int KTHREADS = 320;
-constexpr int KEPI = 4;                // working epilogue warps
-constexpr int KEU = KU / 2;            // units per epilogue thread
+constexpr int KEPI = 4;     // working epilogue warps
 constexpr int XSTAGES = 3;
-constexpr int X_BYTES = KB * KBK * 2;          // 8 KiB: 64 rows x 64 units (SW128)
-constexpr int GATE_BYTES = KU * KBK * 2;       // 4 KiB: one gate's 32 units x 64 K (SW64)
-constexpr int WCHUNK = 4 * GATE_BYTES;         // 16 KiB
-constexpr int SLICE_BYTES = KB * KU * 2;       // 4 KiB: one CTA's h slice (4 k-groups x 64 rows)
-constexpr uint32_t IDESC = make_idesc_bf16_f32(KROWS, KN, false, true);
+constexpr int X_BYTES = KB * KBK * 2;  // 8 KiB: 64 rows x 64 units (SW128)
+
+// Per-CTA slice width KU (hidden units per CTA; the cluster has H / KU CTAs): 32 (8-CTA clusters
+// at H = 256) or 16 (16-CTA clusters: half the MMA and gate math per step — the critical path —
+// for the same DSMEM send volume per CTA).
+template <int KU>
+struct KC {
+    static constexpr int KN = 4 * KU;                         // UMMA N (i | f | o | ĝ)
+    static constexpr int KEU = KU / 2;                        // units per epilogue thread
+    static constexpr int GATE_BYTES = KU * KBK * 2;           // one gate's KU units x 64 K
+    static constexpr int WCHUNK = 4 * GATE_BYTES;             // the 4 gates of one K chunk
+    static constexpr int SLICE_BYTES = KB * KU * 2;           // one CTA's h slice (KU/8 k-groups x 64 rows)
+    static constexpr uint32_t WLAYOUT = KU == 32 ? 4u : 6u;   // SWIZZLE_64B / SWIZZLE_32B (MN-major)
+    static constexpr uint32_t IDESC = make_idesc_bf16_f32(KROWS, KN, false, true);
+    static constexpr int TMEM_COLS = 2 * KN < 32 ? 32 : 2 * KN;
+};
 
 struct KMaps {
     CUtensorMap x, h, W, U;
@@ -87,6 +95,7 @@ struct KLayout {  // byte offsets into the 1024-aligned dynamic shared memory
     int rec0, rec1, xring, w, bars, bias, total;
 };
 
+template <int KU>
 __host__ __device__ constexpr KLayout klayout(int H) {
     KLayout L{};
     const int rec = (H / 8) * 1024;  // H/8 k-groups x 1 KiB
@@ -94,7 +103,7 @@ __host__ __device__ constexpr KLayout klayout(int H) {
     L.rec1 = rec;
     L.xring = 2 * rec;
     L.w = L.xring + XSTAGES * X_BYTES;
-    L.bars = L.w + 2 * (H / KBK) * WCHUNK;
+    L.bars = L.w + 2 * (H / KBK) * KC<KU>::WCHUNK;
     L.bias = L.bars + 256;
     L.total = L.bias + 4 * KU * 4;
     return L;
@@ -116,13 +125,18 @@ __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
 
+template <int KU>
 __global__ void __launch_bounds__(KTHREADS, 1)
 wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
                          const __grid_constant__ KMaps M) {
+    using C = KC<KU>;
+    constexpr int KN = C::KN, KEU = C::KEU, GATE_BYTES = C::GATE_BYTES, WCHUNK = C::WCHUNK;
+    constexpr int SLICE_BYTES = C::SLICE_BYTES;
+    constexpr uint32_t IDESC = C::IDESC;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
     uint8_t* smem = smem_raw + pad;
-    const KLayout L = klayout(P.H);
+    const KLayout L = klayout<KU>(P.H);
     const int KCH = P.H / KBK;           // K chunks per half
     const int CS = P.H / KU;             // CTAs per layer = cluster size
     uint8_t* rec[2] = {smem + L.rec0, smem + L.rec1};
@@ -160,11 +174,11 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
         mbar_arrive_expect_tx(&hfull[0], rec_bytes);
         mbar_arrive_expect_tx(&hfull[1], rec_bytes);
     }
-    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * KU) {  // (4·KU = 128 <= 256 threads past warp 1)
+    if (threadIdx.x >= 64 && threadIdx.x < 64 + 4 * KU) {  // (4·KU <= 128 <= 256 threads past warp 1)
         const int e = threadIdx.x - 64;
         sbias[e] = T.b[(long long)d * 4 * P.H + (e / KU) * P.H + (int)j * KU + e % KU];
     }
-    if (warp == 1) tmem_alloc(tmem_slot, 2 * KN);
+    if (warp == 1) tmem_alloc(tmem_slot, C::TMEM_COLS);
     tc_fence_before();
     __syncthreads();
     cluster_sync();
@@ -212,7 +226,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
         const uint64_t xdesc0 = make_sdesc(smem_u32(xring), 16, 1024);                 // SW128 K-major
         const uint64_t rdesc[2] = {make_sdesc(smem_u32(rec[0]), 1024, 128, 0),         // no swizzle
                                    make_sdesc(smem_u32(rec[1]), 1024, 128, 0)};
-        const uint64_t bdesc0 = make_sdesc(smem_u32(sW), GATE_BYTES, 8 * KU * 2, 4u);   // SW64 MN-major
+        const uint64_t bdesc0 = make_sdesc(smem_u32(sW), GATE_BYTES, 8 * KU * 2, C::WLAYOUT);  // MN-major
         int stage = 0, acc = 0;
         uint32_t phase = 0, acc_phase = 0;
         for (int t = 0; t < P.L0; ++t) {
@@ -287,10 +301,10 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
             uint32_t hp[KEU / 2];
             {
                 float zi[KEU], zf[KEU], zo[KEU], zg[KEU];
-                tmem_ld_32x32b_x16(tbase + 0 * KU, zi);
-                tmem_ld_32x32b_x16(tbase + 1 * KU, zf);
-                tmem_ld_32x32b_x16(tbase + 2 * KU, zo);
-                tmem_ld_32x32b_x16(tbase + 3 * KU, zg);
+                tmem_ld_32x32b<KEU>(tbase + 0 * KU, zi);
+                tmem_ld_32x32b<KEU>(tbase + 1 * KU, zf);
+                tmem_ld_32x32b<KEU>(tbase + 2 * KU, zo);
+                tmem_ld_32x32b<KEU>(tbase + 3 * KU, zg);
                 tmem_wait_ld();
                 tc_fence_before();
                 __syncwarp();
@@ -301,8 +315,8 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
                 //     into every cluster CTA's buffer t & 1, each store carrying complete_tx(16) to
                 //     that CTA's hfull[t & 1] (no staging, no barrier); the next k-group's math
                 //     overlaps those stores in flight
-                const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES + (uint32_t)half * 2048u +
-                                           (uint32_t)row * 16u;
+                const uint32_t dst_local = smem_u32(rec[t & 1]) + j * SLICE_BYTES +
+                                           (uint32_t)half * (KEU / 8) * 1024u + (uint32_t)row * 16u;
                 const uint32_t bar_local = smem_u32(&hfull[t & 1]);
 #pragma unroll
                 for (int g = 0; g < KEU / 8; ++g) {
@@ -379,7 +393,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
     cluster_sync();  // no CTA leaves while a peer may still copy into its shared memory
     if (warp == 1) {
         tc_fence_after();
-        tmem_dealloc(tmem_base, 2 * KN);
+        tmem_dealloc(tmem_base, C::TMEM_COLS);
     }
 }
 
@@ -401,40 +415,61 @@ bool kenc(EncodeTiledFn enc, CUtensorMap* m, int rank, const void* base, const c
     return true;
 }
 
-size_t cluster_smem(int H) { return (size_t)klayout(H).total + 1024; }
+template <int KU>
+size_t cluster_smem(int H) { return (size_t)klayout<KU>(H).total + 1024; }
 
-}  // namespace
-
-// The DSMEM-exchange kernel applies when: stacked LSTM (every dilation 1), batch <= 64, H in
-// {128, 256}, bf16, and the D clusters of H/32 CTAs (one CTA per SM) can all be co-resident.
-bool cluster_kernel_applies(const Problem& p) {
-    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM || p.B > KB || (p.H != 128 && p.H != 256)) return false;
-    for (int d = 0; d < p.D; ++d)
-        if (p.dil[d] != 1) return false;
-    if (cluster_smem(p.H) > 227 * 1024) return false;
-    int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess) return false;
-    cudaFuncSetAttribute(wavefront_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cluster_smem(p.H));
+// Can the D clusters of H / KU CTAs (one per SM) all be co-resident?  (16-CTA clusters need the
+// non-portable cluster size opt-in.)
+template <int KU>
+bool cluster_fits(const Problem& p) {
+    const int cs = p.H / KU;
+    if (cs > 16 || cluster_smem<KU>(p.H) > 227 * 1024) return false;
+    if (cs > 8 && cudaFuncSetAttribute(wavefront_cluster_kernel<KU>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1) !=
+                      cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (cudaFuncSetAttribute(wavefront_cluster_kernel<KU>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)cluster_smem<KU>(p.H)) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)(p.D * (p.H / KU)));
+    cfg.gridDim = dim3((unsigned)(p.D * cs));
     cfg.blockDim = dim3(KTHREADS);
-    cfg.dynamicSmemBytes = cluster_smem(p.H);
+    cfg.dynamicSmemBytes = cluster_smem<KU>(p.H);
     cudaLaunchAttribute a[1];
     a[0].id = cudaLaunchAttributeClusterDimension;
-    a[0].val.clusterDim.x = p.H / KU;
+    a[0].val.clusterDim.x = cs;
     a[0].val.clusterDim.y = 1;
     a[0].val.clusterDim.z = 1;
     cfg.attrs = a;
     cfg.numAttrs = 1;
     int n = 0;
-    if (cudaOccupancyMaxActiveClusters(&n, wavefront_cluster_kernel, &cfg) != cudaSuccess) {
+    if (cudaOccupancyMaxActiveClusters(&n, wavefront_cluster_kernel<KU>, &cfg) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
     return n >= p.D;
 }
 
-cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+// Slice width: 16 units (clusters of H/16 CTAs) when they fit, else 32; 0 = the kernel does not
+// apply.  FT_CLUSTER_UNITS=32|16 forces one (A/B).
+int cluster_units(const Problem& p) {
+    if (p.kind != KIND_SEQ || p.cell != CELL_LSTM || p.B > KB || (p.H != 128 && p.H != 256)) return 0;
+    for (int d = 0; d < p.D; ++d)
+        if (p.dil[d] != 1) return 0;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+    const char* e = getenv("FT_CLUSTER_UNITS");
+    const int want = e ? atoi(e) : 0;
+    if (want != 32 && cluster_fits<16>(p)) return 16;
+    if (want != 16 && cluster_fits<32>(p)) return 32;
+    return 0;
+}
+
+template <int KU>
+cudaError_t launch_cluster_t(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
     void* ptr = nullptr;
     cudaDriverEntryPointQueryResult q = cudaDriverEntryPointSymbolNotFound;
     cudaError_t e = cudaGetDriverEntryPointByVersion("cuTensorMapEncodeTiled", &ptr, 12000, cudaEnableDefault, &q);
@@ -457,15 +492,18 @@ cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStr
         const cuuint32_t box[2] = {KBK, KB};
         if (!kenc(enc, &M.h, 2, t.hb, dims, st, box, CU_TENSOR_MAP_SWIZZLE_128B, err)) return cudaErrorInvalidValue;
     }
-    {  // weights (n, k, gate, layer): (32 units, 64 K, 4 gates, 1) boxes, 64-byte swizzle
+    {  // weights (n, k, gate, layer): (KU units, 64 K, 4 gates, 1) boxes, 64- / 32-byte swizzle
         const cuuint64_t dims[4] = {(cuuint64_t)H, (cuuint64_t)H, 4, (cuuint64_t)p.D};
         const cuuint64_t st[3] = {(cuuint64_t)H * 2, (cuuint64_t)H * H * 2, (cuuint64_t)4 * H * H * 2};
         const cuuint32_t box[4] = {KU, KBK, 4, 1};
-        if (!kenc(enc, &M.W, 4, t.W, dims, st, box, CU_TENSOR_MAP_SWIZZLE_64B, err)) return cudaErrorInvalidValue;
-        if (!kenc(enc, &M.U, 4, t.U, dims, st, box, CU_TENSOR_MAP_SWIZZLE_64B, err)) return cudaErrorInvalidValue;
+        const CUtensorMapSwizzle sw = KU == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+        if (!kenc(enc, &M.W, 4, t.W, dims, st, box, sw, err)) return cudaErrorInvalidValue;
+        if (!kenc(enc, &M.U, 4, t.U, dims, st, box, sw, err)) return cudaErrorInvalidValue;
     }
-    const size_t smem = cluster_smem(H);
-    e = cudaFuncSetAttribute(wavefront_cluster_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    const size_t smem = cluster_smem<KU>(H);
+    e = cudaFuncSetAttribute(wavefront_cluster_kernel<KU>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess && H / KU > 8)
+        e = cudaFuncSetAttribute(wavefront_cluster_kernel<KU>, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
     if (e != cudaSuccess) {
         if (err) *err = std::string("cluster launch setup: ") + cudaGetErrorString(e);
         return e;
@@ -481,12 +519,26 @@ cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStr
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
     int coop = 0;
-    e = launch_cluster_persistent(cfg, attr, 1, &coop, wavefront_cluster_kernel, p, t, M);
+    e = launch_cluster_persistent(cfg, attr, 1, &coop, wavefront_cluster_kernel<KU>, p, t, M);
     if (e == cudaSuccess)
-        set_last_launch("wavefront_cluster_kernel grid=" + std::to_string(p.D * (H / KU)) + " cluster=" +
-                        std::to_string(H / KU) + " cooperative=" + std::to_string(coop));
+        set_last_launch("wavefront_cluster_kernel<" + std::to_string(KU) + "> grid=" + std::to_string(p.D * (H / KU)) +
+                        " cluster=" + std::to_string(H / KU) + " cooperative=" + std::to_string(coop));
     if (e != cudaSuccess && err) *err = std::string("cluster launch: ") + cudaGetErrorString(e);
     return e;
+}
+
+}  // namespace
+
+// The DSMEM-exchange kernel applies when: stacked LSTM (every dilation 1), batch <= 64, H in
+// {128, 256}, bf16, and the D clusters of H/KU CTAs (one CTA per SM) can all be co-resident.
+bool cluster_kernel_applies(const Problem& p) { return cluster_units(p) != 0; }
+
+cudaError_t launch_wavefront_cluster(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
+    const int ku = cluster_units(p);
+    if (ku == 16) return launch_cluster_t<16>(p, t, s, err);
+    if (ku == 32) return launch_cluster_t<32>(p, t, s, err);
+    if (err) *err = "cluster kernel does not apply";
+    return cudaErrorInvalidConfiguration;
 }
 
 }  // namespace ft

@@ -169,6 +169,20 @@ def test_bf16_cluster_dsmem(B, T, H, D, monkeypatch):
     _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"cluster {B,T,H,D}")
 
 
+@pytest.mark.parametrize("units", ["16", "32"])
+@pytest.mark.parametrize("B,T,H,D", [(64, 17, 128, 4), (5, 6, 128, 2)])
+def test_bf16_cluster_slice_widths(B, T, H, D, units, monkeypatch):
+    """The cluster kernel's per-CTA slice: 16 units (H/16 CTAs per cluster; the default whenever
+    those clusters fit — H = 128) or 32 units.  Both against the oracle, and the launch really
+    used the requested slice."""
+    monkeypatch.setenv("FT_CLUSTER", "1")
+    monkeypatch.setenv("FT_CLUSTER_UNITS", units)
+    p = ftgen.stacked_inputs(B, T, H, D, 5150 + B + D, "bf16")
+    got = _run_stacked(p, torch.bfloat16, want_all=True)
+    assert f"wavefront_cluster_kernel<{units}>" in ft.ft_last_launch(), ft.ft_last_launch()
+    _check(got, _oracle_stacked(p, want_all=True), torch.bfloat16, ALL, ctx=f"cluster KU={units} {B,T,H,D}")
+
+
 def test_bf16_cluster_stress_and_repeat(monkeypatch):
     """Random release delays on the depth edge (stress mode) and repeated calls on one workspace:
     results bitwise identical run to run."""
