@@ -351,7 +351,7 @@ int hostio_chunk() {
 }
 
 struct HostIoPlan {
-    size_t x_off, y_off, hn_off, cn_off, ysig_off, xsig_off, inner_off, total;
+    size_t x_off, y_off, hn_off, cn_off, ysig_off, xsig_off, nsig_off, inner_off, total;
     int nchunks;
 };
 HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, size_t inner) {
@@ -364,7 +364,8 @@ HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, s
     h.cn_off = h.hn_off + round_up((size_t)batch * depth * hidden * es, 256);
     h.ysig_off = h.cn_off + round_up((size_t)batch * depth * hidden * 4, 256);
     h.xsig_off = h.ysig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
-    h.inner_off = h.xsig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
+    h.nsig_off = h.xsig_off + round_up((size_t)h.nchunks * sizeof(int), 256);
+    h.inner_off = h.nsig_off + round_up((size_t)depth * sizeof(int), 256);
     h.total = h.inner_off + inner;
     return h;
 }
@@ -374,9 +375,10 @@ HostIoPlan plan_hostio(int batch, int seq, int hidden, int depth, ft_dtype dt, s
 // counters).  The two events are created per call and released once enqueued (re-entrancy).
 struct HostIoStreams {
     cudaStream_t copy = nullptr;  // device→host y chunks (waits on the kernel's counters)
+    cudaStream_t state = nullptr; // device→host h_n / c_n per layer (waits on the kernel's counters)
     cudaStream_t h2d = nullptr;   // host→device x chunks (never waits on a kernel: no cycle
                                   // between concurrent calls sharing the streams)
-    cudaEvent_t reset = nullptr, done = nullptr, xdone = nullptr;
+    cudaEvent_t reset = nullptr, done = nullptr, xdone = nullptr, sdone = nullptr;
 };
 typedef CUresult (*StreamWaitValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
 typedef CUresult (*StreamWriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
@@ -405,15 +407,17 @@ bool hostio_streams(HostIoStreams* out, StreamWaitValue32Fn* wait_fn, StreamWrit
     }
     HostIoStreams& h = per_dev[dev];
     if (!h.copy && (cudaStreamCreateWithFlags(&h.copy, cudaStreamNonBlocking) != cudaSuccess ||
-                    cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking) != cudaSuccess)) {
+                    cudaStreamCreateWithFlags(&h.h2d, cudaStreamNonBlocking) != cudaSuccess ||
+                    cudaStreamCreateWithFlags(&h.state, cudaStreamNonBlocking) != cudaSuccess)) {
         cudaGetLastError();
-        h.copy = h.h2d = nullptr;
+        h.copy = h.h2d = h.state = nullptr;
         return false;
     }
     *out = h;
     if (cudaEventCreateWithFlags(&out->reset, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreateWithFlags(&out->done, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&out->xdone, cudaEventDisableTiming) != cudaSuccess) {
+        cudaEventCreateWithFlags(&out->xdone, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&out->sdone, cudaEventDisableTiming) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
@@ -492,7 +496,8 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
         t.ysig_per_chunk = &per_chunk;
         t.xsig = reinterpret_cast<int*>(ws + hp.xsig_off);
         t.xchunk = chunk;
-        e = cudaMemsetAsync(t.ysig, 0, (size_t)(hp.xsig_off - hp.ysig_off) + (size_t)hp.nchunks * sizeof(int), s);
+        t.nsig = reinterpret_cast<int*>(ws + hp.nsig_off);
+        e = cudaMemsetAsync(t.ysig, 0, (size_t)(hp.nsig_off - hp.ysig_off) + (size_t)depth * sizeof(int), s);
         if (e == cudaSuccess) e = cudaEventRecord(hs.reset, s);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(hs.h2d, hs.reset, 0);
         const size_t row = (size_t)seq * hidden * es;
@@ -510,6 +515,7 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
             cudaEventDestroy(hs.reset);
             cudaEventDestroy(hs.done);
             cudaEventDestroy(hs.xdone);
+            cudaEventDestroy(hs.sdone);
             return fail(FT_ERR_CUDA, std::string("hostio setup: ") + cudaGetErrorString(e));
         }
     } else {
@@ -523,8 +529,35 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
             cudaEventDestroy(hs.reset);
             cudaEventDestroy(hs.done);
             cudaEventDestroy(hs.xdone);
+            cudaEventDestroy(hs.sdone);
         }
         return st;
+    }
+    // h_n / c_n per layer as soon as the layer's last step is stored (nsig counters): layers of
+    // earlier bands leave the device while the later bands still run
+    bool state_overlapped = false;
+    if (per_step > 0) {
+        cudaError_t se = cudaStreamWaitEvent(hs.state, hs.reset, 0);
+        const size_t hrow = (size_t)hidden * es, crow = (size_t)hidden * 4;
+        const size_t hpitch = (size_t)depth * hrow, cpitch = (size_t)depth * crow;
+        for (int d = 0; d < depth && se == cudaSuccess; ++d) {
+            if (wait_value(hs.state, (CUdeviceptr)(t.nsig + d), (cuuint32_t)per_step, CU_STREAM_WAIT_VALUE_GEQ) !=
+                CUDA_SUCCESS) {
+                se = cudaErrorUnknown;
+                break;
+            }
+            se = cudaMemcpy2DAsync(static_cast<uint8_t*>(h_n_host) + d * hrow, hpitch, ws + hp.hn_off + d * hrow,
+                                   hpitch, hrow, batch, cudaMemcpyDeviceToHost, hs.state);
+            if (se == cudaSuccess)
+                se = cudaMemcpy2DAsync(reinterpret_cast<uint8_t*>(c_n_host) + d * crow, cpitch,
+                                       ws + hp.cn_off + d * crow, cpitch, crow, batch, cudaMemcpyDeviceToHost,
+                                       hs.state);
+        }
+        state_overlapped = se == cudaSuccess;
+        if (!state_overlapped) cudaGetLastError();  // fall back below: copy after the kernel on `s`
+        // `s` waits for whatever the state stream enqueued (also on the fallback path)
+        if (cudaEventRecord(hs.sdone, hs.state) == cudaSuccess) cudaStreamWaitEvent(s, hs.sdone, 0);
+        else state_overlapped = false;
     }
     if (per_step > 0) {
         e = cudaStreamWaitEvent(hs.copy, hs.reset, 0);
@@ -553,9 +586,12 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
         cudaEventDestroy(hs.reset);
         cudaEventDestroy(hs.done);
         cudaEventDestroy(hs.xdone);
+        cudaEventDestroy(hs.sdone);
     }
-    if (e == cudaSuccess) e = cudaMemcpyAsync(h_n_host, ws + hp.hn_off, hb, cudaMemcpyDeviceToHost, s);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);
+    if (!state_overlapped) {
+        if (e == cudaSuccess) e = cudaMemcpyAsync(h_n_host, ws + hp.hn_off, hb, cudaMemcpyDeviceToHost, s);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(c_n_host, ws + hp.cn_off, cb, cudaMemcpyDeviceToHost, s);
+    }
     if (e != cudaSuccess) return fail(FT_ERR_CUDA, std::string("D2H: ") + cudaGetErrorString(e));
     return FT_OK;
 }

@@ -48,6 +48,10 @@ struct Tensors {
     int ychunk = 0;
     int* ysig_per_step = nullptr;  // HOST: set by the launcher to the increments per time step
                                    // (0 = this launch does not signal; copy y after the kernel)
+    // host-IO overlap of the final states: after storing its share of h_n / c_n (cell (d, T-1)),
+    // every epilogue warp fences at system scope and adds 1 to nsig[d]; a second copy stream
+    // moves layer d's rows to the host once nsig[d] reaches *ysig_per_step (same count per cell)
+    int* nsig = nullptr;
     int* ysig_per_chunk = nullptr; // HOST: 1 = owner walk: each warp signals once per chunk (its
                                    // last step of the chunk), so a chunk completes at per_step
 };

@@ -756,6 +756,15 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                     d4[v] = make_float4(cst[4 * v], cst[4 * v + 1], cst[4 * v + 2], cst[4 * v + 3]);
             }
         }
+        // host-IO overlap: this warp's share of layer d's final state is stored → fence at system
+        // scope (a copy engine reads it) and count it for the state copy stream (ft_api.cu hostio)
+        if (last && T.nsig) {
+            __syncwarp();
+            if (lane == 0) {
+                fence_acq_rel_sys();
+                red_relaxed_sys_add(T.nsig + c.d, 1);
+            }
+        }
         // (4) host-IO overlap: this warp's share of y(·, t, ·) is stored → fence at system scope
         //     (a copy engine reads it) and count it for the copy stream (ft_api.cu hostio)
         if (top && T.ysig && (P.owner != 1 || c.i % T.ychunk == T.ychunk - 1 || c.i == P.L0 - 1)) {
