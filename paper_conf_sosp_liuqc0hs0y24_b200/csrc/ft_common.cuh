@@ -370,13 +370,10 @@ struct TileWalk {
                            // non-layer-0 tiles, and that index of the current cell's first tile
 };
 
-// PAIRS = false compiles the cell-pair branch out (kernels that never run cell pairs keep their
-// walk state small: no PairCursor in registers).
-template <bool PAIRS = true>
 FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
     TileWalk w;
     w.cur = cursor_begin();
-    if (PAIRS && p.cpair) w.pc = pair_begin(p);
+    if (p.cpair) w.pc = pair_begin(p);
     w.tile = worker;
     w.stride = nworkers;
     w.e = -1;
@@ -401,9 +398,8 @@ FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
     return w;
 }
 
-template <bool PAIRS = true>
 FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) {
-    if (PAIRS && p.cpair) {  // round-robin over the pair tiles
+    if (p.cpair) {  // round-robin over the pair tiles
         if (w.tile >= p.ntiles) return false;
         tl = decode_pair_tile(p, w.pc, w.tile);
         tid = w.tile;

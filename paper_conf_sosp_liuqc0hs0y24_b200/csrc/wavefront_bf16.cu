@@ -213,7 +213,7 @@ __global__ void pack_rows_kernel(const __nv_bfloat16* __restrict__ src, __nv_bfl
 // full barrier (in the leader CTA) takes one expect-tx arrival from each of the leader's two
 // producers; the peer CTA's producers only issue loads.  Splitting halves the serial TMA issue
 // work per thread (the role trace showed one thread issuing both was the limiter).
-template <int CG, int U, bool kWeights, bool PR = false>
+template <int CG, int U, bool kWeights>
 __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T, const Maps& M,
                                              uint8_t* sA, uint8_t* sB, uint64_t* full,
                                              uint64_t* empty, uint32_t rank) {
@@ -230,24 +230,24 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     if (P.l2pol & 3) pol_stream = pol_keep = l2_policy(P.l2pol & 3, pol_keep);
     const bool skipB = FT_DEV_BIT(P.debug, 16), fixed = FT_DEV_BIT(P.debug, 32);  // timing experiments
     const uint32_t tx = kWeights ? (skipB ? 0 : CG * C::B_BYTES) : CG * C::A_BYTES;
-    TileWalk walk = walk_begin<PR>(P, blockIdx.x / CG, gridDim.x / CG);
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     FT_TR_ROLE;
     TileId tl;
     long long tile;
-    while (walk_next<PR>(P, walk, tl, tile)) {
-        // (PR && P.cpair): this CTA's own cell (rank 1 takes the pair's second cell, or idles when the
+    while (walk_next(P, walk, tl, tile)) {
+        // P.cpair: this CTA's own cell (rank 1 takes the pair's second cell, or idles when the
         // group had an odd count); every pair tile runs all three K segments, a segment a cell
         // lacks (its zero boundary state) reading an all-zero block
         TileId tm = tl;
         bool mine = true;
-        if ((PR && P.cpair) && rank == 1) {
+        if (P.cpair && rank == 1) {
             tm.cell = tl.cell2;
             mine = tl.has2 != 0;
         }
         Segment seg[3];
         const int ns = segments(P, kWeights ? tl : tm, seg);
-        const int nchunks = ((PR && P.cpair) ? 3 : ns) * kchunks;
-        const int arow0 = (PR && P.cpair) ? 0 : tl.m * ROWS * CG + (int)rank * ROWS;
+        const int nchunks = (P.cpair ? 3 : ns) * kchunks;
+        const int arow0 = P.cpair ? 0 : tl.m * ROWS * CG + (int)rank * ROWS;
         const bool lin = P.cell == CELL_LINEAR;
         const int bn = (fixed || lin) ? 0 : tl.n * U;
         const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
@@ -297,12 +297,12 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                     tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
                                               fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
                 }
-            } else if ((PR && P.cpair) && (!mine || sg.src == SRC_NONE)) {
+            } else if (P.cpair && (!mine || sg.src == SRC_NONE)) {
                 tma_load_2d_hint_addr<CG>(sA0 + (uint32_t)(stage * C::A_BYTES), &M.h, bar, 0, P.zrow, pol_act);
             } else {
                 load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
             }
-            if (++kc == kchunks) { kc = 0; si = (PR && P.cpair) ? si + 1 : next_segment(seg, si); }
+            if (++kc == kchunks) { kc = 0; si = P.cpair ? si + 1 : next_segment(seg, si); }
             if (++stage == C::STAGES) {
                 stage = 0;
                 phase ^= 1;
@@ -315,7 +315,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
 }
 
 // ------------------------------------------------------------------------------ MMA issuer
-template <int CG, int U, bool PR = false>
+template <int CG, int U>
 __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, uint8_t* sA,
                                         uint8_t* sB, uint64_t* full, uint64_t* empty,
                                         uint64_t* tfull, uint64_t* tempty) {
@@ -330,13 +330,13 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
     //    8*WROW apart (SBO); K step of 16 rows = 16*WROW.  CG 2: each CTA holds half the atoms.
     const uint64_t adesc0 = make_sdesc(smem_u32(sA), 16, 1024);
     const uint64_t bdesc0 = make_sdesc(smem_u32(sB), U * BK * 2, 8 * C::WROW, C::WLAYOUT);
-    TileWalk walk = walk_begin<PR>(P, blockIdx.x / CG, gridDim.x / CG);
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     FT_TR_ROLE;
     TileId tl;
     long long tile;
-    while (walk_next<PR>(P, walk, tl, tile)) {
+    while (walk_next(P, walk, tl, tile)) {
         Segment seg[3];
-        const int nchunks = ((PR && P.cpair) ? 3 : segments(P, tl, seg)) * kchunks;
+        const int nchunks = (P.cpair ? 3 : segments(P, tl, seg)) * kchunks;
         FT_TR_DECL;
         FT_TR_BEGIN();
         mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
@@ -413,7 +413,6 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
                                                     uint32_t tmem_base, uint64_t* tfull,
                                                     uint64_t* tempty, uint32_t rank) {
     using C = KCfg<CG, U>;
-    constexpr bool PR = false;  // the linear cell never runs cell pairs
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int q = warp & 3, half = (warp - 2) >> 2, row = q * 32 + lane;
     constexpr int COLS = 4 * U / EPI_PARTS;  // accumulator columns per warp
@@ -422,10 +421,10 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
     uint32_t acc_phase = 0;
     const int target = flag_target(P);
     __nv_bfloat16* ys = (__nv_bfloat16*)T.h_all;
-    TileWalk walk = walk_begin<PR>(P, blockIdx.x / CG, gridDim.x / CG);
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     TileId tl;
     long long tile;
-    while (walk_next<PR>(P, walk, tl, tile)) {
+    while (walk_next(P, walk, tl, tile)) {
         const Cell c = tl.cell;
         int ci = 0, cj = 0;
         const long long cprod = c_producer(P, tl, &ci, &cj);
@@ -492,7 +491,7 @@ __device__ __forceinline__ void run_epilogue_linear(const Problem& P, const Tens
     }
 }
 
-template <int CG, int U, bool PR = false>
+template <int CG, int U>
 __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T, uint32_t tmem_base,
                                              uint64_t* tfull, uint64_t* tempty, uint32_t rank,
                                              float* sbias) {
@@ -516,7 +515,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     __nv_bfloat16* h_all = (__nv_bfloat16*)T.h_all;
     __nv_bfloat16* y = (__nv_bfloat16*)T.y;
     __nv_bfloat16* h_n = (__nv_bfloat16*)T.h_n;
-    TileWalk walk = walk_begin<PR>(P, blockIdx.x / CG, gridDim.x / CG);
+    TileWalk walk = walk_begin(P, blockIdx.x / CG, gridDim.x / CG);
     // L2 priority of the nest's live state (the c ring and the blocked h): EVICT_LAST, so the
     // EVICT_FIRST weight stream does not push it out before the next diagonal reads it (ncu, C3:
     // DRAM 30.8 -> 30.1 GB per launch).  FT_DEBUG bit 128 (development builds) reverts to EVICT_NORMAL.
@@ -534,17 +533,17 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     FT_TR_ROLE;
     TileId tl;
     long long tile;
-    while (walk_next<PR>(P, walk, tl, tile)) {
-        TileId tm = tl;  // this CTA's cell ((PR && P.cpair): rank 1 takes the pair's second cell)
+    while (walk_next(P, walk, tl, tile)) {
+        TileId tm = tl;  // this CTA's cell (P.cpair: rank 1 takes the pair's second cell)
         bool mine = true;
-        if ((PR && P.cpair) && rank == 1) {
+        if (P.cpair && rank == 1) {
             tm.cell = tl.cell2;
             mine = tl.has2 != 0;
         }
         const Cell c = tm.cell;
         int ci = 0, cj = 0;
         const long long cprod = mine ? c_producer(P, tm, &ci, &cj) : -1;
-        const int b = (PR && P.cpair) ? row : tl.m * ROWS * CG + (int)rank * ROWS + row;
+        const int b = P.cpair ? row : tl.m * ROWS * CG + (int)rank * ROWS + row;
         const bool valid = mine && b < P.B;
         const int n0 = tl.n * U + half * EPI_UNITS;
         FT_TR_DECL;
@@ -800,7 +799,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     FT_TR_FLUSH(leader_thread);
 }
 
-template <int CG, int U, bool PR = false>
+template <int CG, int U>
 __global__ void __launch_bounds__(THREADS, 1)
 wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
                       const __grid_constant__ Maps M) {
@@ -847,13 +846,13 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     const uint32_t tmem_base = *tmem_slot;
 
     if (warp == 0) {
-        if (lane == 0) run_producer<CG, U, true, PR>(P, T, M, sA, sB, full, empty, rank);
+        if (lane == 0) run_producer<CG, U, true>(P, T, M, sA, sB, full, empty, rank);
     } else if (warp == 1) {
-        if (rank == 0) run_mma<CG, U, PR>(P, tmem_base, sA, sB, full, empty, tfull, tempty);  // whole warp
+        if (rank == 0) run_mma<CG, U>(P, tmem_base, sA, sB, full, empty, tfull, tempty);  // whole warp
     } else if (warp == ACT_WARP) {
-        if (lane == 0) run_producer<CG, U, false, PR>(P, T, M, sA, sB, full, empty, rank);
+        if (lane == 0) run_producer<CG, U, false>(P, T, M, sA, sB, full, empty, rank);
     } else {
-        run_epilogue<CG, U, PR>(P, T, tmem_base, tfull, tempty, rank, sbias);
+        run_epilogue<CG, U>(P, T, tmem_base, tfull, tempty, rank, sbias);
     }
 
     tc_fence_before();
@@ -1084,7 +1083,7 @@ cudaError_t encode_maps(const Problem& p, const Tensors& t, EncodeTiledFn enc, b
     return cudaSuccess;
 }
 
-template <int CG, int U, bool PR>
+template <int CG, int U>
 cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err,
                            const Maps& M, bool x_direct, int dev, int nsm, int* clusters) {
     using C = KCfg<CG, U>;
@@ -1130,7 +1129,7 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
         cfg.numAttrs = 1;
         int nclusters = clusters[dev];
         if (nclusters < 1) {
-            e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U, PR>, &cfg);
+            e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U>, &cfg);
             if (e != cudaSuccess || nclusters < 1) {
                 if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
                 return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
@@ -1229,10 +1228,10 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
     }
     int coop = 1;
     if constexpr (CG == 2)
-        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, &coop, wavefront_bf16_kernel<CG, U, PR>,
+        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, &coop, wavefront_bf16_kernel<CG, U>,
                                       q, t, M);
     else
-        e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U, PR>, q, t, M);
+        e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
     if (e == cudaSuccess)
         set_last_launch("wavefront_bf16_kernel<" + std::to_string(CG) + "," + std::to_string(U) +
                         "> grid=" + std::to_string(grid) + " cluster=" + std::to_string(CG) +
@@ -1246,7 +1245,7 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
     return e;
 }
 
-template <int CG, int U, bool PR = false>
+template <int CG, int U>
 cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err) {
     using C = KCfg<CG, U>;
     EncodeTiledFn enc = get_encode_fn(err);
@@ -1274,7 +1273,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     static bool attr_set[64] = {};
     static int clusters[64] = {};
     if (!attr_set[dev]) {
-        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U, PR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  C::SMEM_BYTES);
         if (e != cudaSuccess) {
             if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
@@ -1282,7 +1281,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         }
         attr_set[dev] = true;
     }
-    return launch_cg_maps<CG, U, PR>(p, t, s, err, M, x_direct, dev, nsm, clusters);
+    return launch_cg_maps<CG, U>(p, t, s, err, M, x_direct, dev, nsm, clusters);
 }
 
 }  // namespace
@@ -1378,8 +1377,7 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
     if (const char* env = getenv("FT_TILE_UNITS")) units = atoi(env) == 32 && p.cell == CELL_LSTM ? 32 : 64;
     if (pp.cpair) units = 64;
     if (units == 64)
-        return cg == 2 ? (pp.cpair ? launch_cg<2, 64, true>(pp, t, s, err) : launch_cg<2, 64>(pp, t, s, err))
-                       : launch_cg<1, 64>(p, t, s, err);
+        return cg == 2 ? launch_cg<2, 64>(pp, t, s, err) : launch_cg<1, 64>(p, t, s, err);
     Problem q = p;
     q.BNU = 32;
     q.NT = p.H / 32;
