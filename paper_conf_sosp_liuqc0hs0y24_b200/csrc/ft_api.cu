@@ -852,35 +852,3 @@ FT_API long long ft_ssa_slots(int depth, int seq, const int* dilations, int band
     }
     return rows;
 }
-
-FT_API long long ft_grid_cell_pairs(int depth, int len_x, int len_y, int band, int* out, long long cap) {
-    if (depth <= 0 || len_x <= 0 || len_y <= 0 || depth > FT_MAX_DEPTH || (cap > 0 && !out)) return -1;
-    ft::Problem p;
-    std::memset(&p, 0, sizeof(p));
-    p.kind = ft::KIND_GRID;
-    p.D = depth;
-    p.L0 = len_x;
-    p.L1 = len_y;
-    p.naxes = 2;
-    p.MB = p.NT = 1;
-    p.ncells = (long long)depth * len_x * len_y;
-    p.band = band > 0 && band < depth ? band : 0;
-    p.cpair = 1;
-    ft::PairCursor c = ft::pair_begin(p);
-    long long n = 0;
-    for (;;) {
-        if (n < cap) {
-            int* o = out + 6 * n;
-            o[0] = c.a.k;
-            o[1] = c.a.d;
-            o[2] = c.a.i;
-            o[3] = c.a.j;
-            o[4] = c.hasb ? c.b.i : -1;
-            o[5] = c.hasb ? c.b.j : -1;
-        }
-        ++n;
-        if (c.nxt.d >= p.D) break;
-        ft::pair_fill(p, c);
-    }
-    return n;
-}

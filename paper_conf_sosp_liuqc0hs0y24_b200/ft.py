@@ -34,7 +34,6 @@ EXPORTS = (
     "ft_dilated_rnn_workspace_size", "ft_dilated_rnn_fwd",
     "ft_grid_rnn_workspace_size", "ft_grid_rnn_fwd",
     "ft_wavefront_cells", "ft_wavefront_cells_banded", "ft_tile_walk", "ft_ssa_slots",
-    "ft_grid_cell_pairs",
     "ft_comm_create", "ft_comm_gather", "ft_comm_destroy",
     "ft_comm_unique_id", "ft_comm_init_rank", "ft_comm_gather_rank",
     "ft_ipc_export", "ft_ipc_open", "ft_ipc_close",
@@ -137,8 +136,6 @@ def lib():
         L.ft_wavefront_cells_banded.restype = _c_ll
         L.ft_wavefront_cells_banded.argtypes = [_c_int] * 6 + [_c_vp, _c_ll]
         L.ft_tile_walk.restype = _c_ll
-        L.ft_grid_cell_pairs.restype = _c_ll
-        L.ft_grid_cell_pairs.argtypes = [_c_int] * 4 + [_c_vp, _c_ll]
         L.ft_ssa_slots.restype = _c_ll
         L.ft_ssa_slots.argtypes = [_c_int, _c_int, _c_vp, _c_int, _c_vp, _c_vp]
         L.ft_tile_walk.argtypes = [_c_int] * 8 + [_c_vp, _c_ll]
@@ -285,16 +282,6 @@ def ft_ssa_slots(depth, seq, dilations, band):
     if rows < 0:
         raise FTError(FT_ERR_INVALID_ARGUMENT, "bad ssa-slot query")
     return rows, list(off), list(mask)
-
-
-def ft_grid_cell_pairs(depth, len_x, len_y, band=0):
-    """[(diagonal, d, i_a, j_a, i_b, j_b), ...] of the grid kernel's cell pairs — host only."""
-    n = lib().ft_grid_cell_pairs(depth, len_x, len_y, band, None, 0)
-    if n < 0:
-        raise FTError(FT_ERR_INVALID_ARGUMENT, "bad cell-pair query")
-    buf = (ctypes.c_int * (6 * n))()
-    lib().ft_grid_cell_pairs(depth, len_x, len_y, band, ctypes.cast(buf, _c_vp), n)
-    return [tuple(buf[6 * k:6 * k + 6]) for k in range(n)]
 
 
 def ft_comm_create(devices):

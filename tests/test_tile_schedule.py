@@ -355,27 +355,3 @@ def test_ssa_ring_layout_sizes():
     assert [m for m in mask].count(-1) == 3  # the boundary layers of bands 0..2
     rows, off, mask = ft.ft_ssa_slots(6, 100, [1, 2, 4, 8, 16, 32], 0)  # C4
     assert mask == [3, 3, 7, 15, 31, 63]
-
-
-# ------------------------------------------------------------------ grid cell pairs (C5)
-@pytest.mark.parametrize("D,Lx,Ly,band", [(4, 32, 32, 1), (3, 5, 7, 0), (2, 1, 6, 0), (4, 6, 3, 2), (1, 4, 4, 0)])
-def test_grid_cell_pairs_cover_and_respect_dependences(D, Lx, Ly, band):
-    """The bf16 grid kernel runs two cells of one (diagonal, depth) group per CTA pair.  Every
-    cell appears exactly once; both cells of a pair share depth and diagonal; every producer of
-    either cell (Table 4: e_depth, e_x, e_y) lies in an EARLIER pair — the wavefront order and
-    its deadlock freedom carry over to the pairs."""
-    pairs = ft.ft_grid_cell_pairs(D, Lx, Ly, band)
-    pos = {}
-    for idx, (k, d, ia, ja, ib, jb) in enumerate(pairs):
-        for (i, j) in ((ia, ja),) + (((ib, jb),) if ib >= 0 else ()):
-            assert (d, i, j) not in pos
-            pos[(d, i, j)] = idx
-        if ib >= 0:
-            assert ia + ja == ib + jb  # same diagonal of the same depth
-    assert len(pos) == D * Lx * Ly
-    for (d, i, j), idx in pos.items():
-        for prod in ((d - 1, i, j), (d, i - 1, j), (d, i, j - 1)):
-            if prod in pos:
-                assert pos[prod] < idx, ((d, i, j), prod)
-    full = sum(1 for p in pairs if p[4] >= 0)
-    assert full >= (len(pos) - len(pairs)) and 2 * full + (len(pairs) - full) == len(pos)
