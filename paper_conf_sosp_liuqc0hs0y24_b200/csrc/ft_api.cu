@@ -136,10 +136,8 @@ WsPlan plan_workspace(const ft::Problem& p, ft_dtype dt, bool h_all_provided) {
     w.ring_off = w.flags_off + w.flags_bytes;
     w.ring_bytes = round_up((size_t)ft::c_ring_elems(p) * sizeof(float), 256);
     w.hall_off = w.ring_off + w.ring_bytes;
-    if (dt == FT_BF16)  // the blocked SSA activation buffer (full, or per-layer rings: p.hring);
-                        // grid nests: + one all-zero K-chunk block (cell-pair tiles)
-        w.hall_bytes = round_up(((size_t)ft::hb_rows_total(p) +
-                                 (p.kind == ft::KIND_GRID ? (size_t)p.MB * p.BM : 0)) * 64 * 2, 256);
+    if (dt == FT_BF16)  // the blocked SSA activation buffer (full, or per-layer rings: p.hring)
+        w.hall_bytes = round_up((size_t)ft::hb_rows_total(p) * 64 * 2, 256);
     else
         w.hall_bytes = h_all_provided
                            ? 0

@@ -63,11 +63,6 @@ struct Problem {
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
-    int cpair;           // bf16 KIND_GRID on CTA pairs: the two CTAs of a pair take two cells of
-                         // the same (diagonal, depth) group — one cell each — and share the weight
-                         // tile (see PairCursor); 0 = one cell per tile
-    int zrow;            // cpair: first row of an all-zero K-chunk block in hb (A of a missing
-                         // segment: boundary cells, or the idle CTA of an odd group)
     int hring;           // bf16 streaming KIND_SEQ: hb holds a ring of slots per layer instead of
                          // every (d, t) row (see hb_slot_row); 0 = one row per (d, t)
     int hb_rows;         // hring: rows of hb the workspace reserves (Σ ring lengths + 2·L0)
@@ -253,8 +248,6 @@ FT_HD void cursor_seek(const Problem& p, Cursor& cur, long long target_ord) {
 struct TileId {
     Cell cell;
     int axis, m, n;
-    Cell cell2;  // p.cpair: the cell of the pair's second CTA (valid when has2)
-    int has2;
 };
 
 FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
@@ -267,8 +260,6 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
     int w = (int)(tile - cur.tile0);
     TileId t;
     t.cell = cur.cell;
-    t.cell2 = cur.cell;
-    t.has2 = 0;
     t.axis = 0;
     t.m = 0;
     if (p.naxes == 1 && p.MB == 1) {  // the common case: the within-cell index is the N-tile
@@ -279,67 +270,6 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
     w /= p.NT;
     t.m = w % p.MB;
     t.axis = w / p.MB;
-    return t;
-}
-
-// Cell pairs (p.cpair, grid nests whose batch fits one 128-row CTA): the cells of one (diagonal,
-// depth) group — consecutive in next_cell order — are taken two at a time, one per CTA of a
-// tcgen05 CTA pair, so the pair's M = 256 MMA computes both cells against ONE weight tile (same
-// depth and axis); the last cell of an odd group runs with an idle partner.  Both cells of a pair
-// lie on one diagonal, so every producer of either cell is in an earlier pair: the wavefront
-// order, and its deadlock-freedom argument, carry over.
-struct PairCursor {
-    long long ord, tile0;  // pair ordinal and its first tile
-    Cell a, b, nxt;        // the pair's cells (b valid when hasb) and the next unpaired cell
-    int hasb;
-};
-FT_HD bool same_group(const Cell& x, const Cell& y) { return x.k == y.k && x.d == y.d; }
-FT_HD void pair_fill(const Problem& p, PairCursor& c) {
-    c.a = c.nxt;
-    const Cell n = next_cell(p, c.a);
-    if (n.d < p.D && same_group(c.a, n)) {
-        c.b = n;
-        c.hasb = 1;
-        c.nxt = next_cell(p, n);
-    } else {
-        c.b = c.a;
-        c.hasb = 0;
-        c.nxt = n;
-    }
-}
-FT_HD PairCursor pair_begin(const Problem& p) {
-    PairCursor c;
-    c.ord = 0;
-    c.tile0 = 0;
-    c.nxt = first_cell();
-    pair_fill(p, c);
-    return c;
-}
-// Number of pairs of the whole nest (host: sizes the tile count).
-inline long long count_pairs(const Problem& p) {
-    PairCursor c = pair_begin(p);
-    long long n = 1;
-    while (c.nxt.d < p.D) {
-        pair_fill(p, c);
-        ++n;
-    }
-    return n;
-}
-FT_HD TileId decode_pair_tile(const Problem& p, PairCursor& cur, long long tile) {
-    const int tpc = p.naxes * p.NT;  // one m-block
-    while (tile >= cur.tile0 + tpc) {
-        pair_fill(p, cur);
-        ++cur.ord;
-        cur.tile0 += tpc;
-    }
-    const int w = (int)(tile - cur.tile0);
-    TileId t;
-    t.cell = cur.a;
-    t.cell2 = cur.b;
-    t.has2 = cur.hasb;
-    t.m = 0;
-    t.n = w % p.NT;
-    t.axis = w / p.NT;
     return t;
 }
 
@@ -363,7 +293,6 @@ FT_HD TileId decode_pair_tile(const Problem& p, PairCursor& cur, long long tile)
 //    of the global order).
 struct TileWalk {
     Cursor cur;
-    PairCursor pc;  // p.cpair
     long long tile, stride;
     int e, n, d0, t;     // owner modes (e < 0: idle worker; e == -2: round-robin rest)
     long long next, idx0;  // p.owner == 2, the rest: next tile index of this worker among the
@@ -373,7 +302,6 @@ struct TileWalk {
 FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
     TileWalk w;
     w.cur = cursor_begin();
-    if (p.cpair) w.pc = pair_begin(p);
     w.tile = worker;
     w.stride = nworkers;
     w.e = -1;
@@ -399,13 +327,6 @@ FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
 }
 
 FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) {
-    if (p.cpair) {  // round-robin over the pair tiles
-        if (w.tile >= p.ntiles) return false;
-        tl = decode_pair_tile(p, w.pc, w.tile);
-        tid = w.tile;
-        w.tile += w.stride;
-        return true;
-    }
     if (!p.owner) {
         if (w.tile >= p.ntiles) return false;
         tl = decode_tile(p, w.cur, w.tile);
@@ -419,8 +340,6 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
             if (w.cur.cell.d != 0) {
                 if (w.next < w.idx0 + tpc) {
                     tl.cell = w.cur.cell;
-                    tl.cell2 = tl.cell;
-                    tl.has2 = 0;
                     tl.axis = 0;
                     tl.m = 0;
                     tl.n = (int)(w.next - w.idx0);
@@ -439,8 +358,6 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
     if (p.owner == 2) {  // layer-0 owner
         if (w.e != 0 || w.t >= p.L0) return false;
         tl.cell = Cell{w.t, 0, w.t, 0, 0, w.t};
-        tl.cell2 = tl.cell;
-        tl.has2 = 0;
         tl.axis = 0;
         tl.m = 0;
         tl.n = w.n;
@@ -455,7 +372,6 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
         w.t = 0;
     }
     if (w.d0 >= p.D) return false;
-    tl.has2 = 0;
     tl.cell.d = w.d0 + w.e;
     tl.cell.i = w.t;
     tl.cell.j = 0;

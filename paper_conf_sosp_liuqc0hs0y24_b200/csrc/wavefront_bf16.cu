@@ -235,19 +235,10 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     TileId tl;
     long long tile;
     while (walk_next(P, walk, tl, tile)) {
-        // P.cpair: this CTA's own cell (rank 1 takes the pair's second cell, or idles when the
-        // group had an odd count); every pair tile runs all three K segments, a segment a cell
-        // lacks (its zero boundary state) reading an all-zero block
-        TileId tm = tl;
-        bool mine = true;
-        if (P.cpair && rank == 1) {
-            tm.cell = tl.cell2;
-            mine = tl.has2 != 0;
-        }
         Segment seg[3];
-        const int ns = segments(P, kWeights ? tl : tm, seg);
-        const int nchunks = (P.cpair ? 3 : ns) * kchunks;
-        const int arow0 = P.cpair ? 0 : tl.m * ROWS * CG + (int)rank * ROWS;
+        const int ns = segments(P, tl, seg);
+        const int nchunks = ns * kchunks;
+        const int arow0 = tl.m * ROWS * CG + (int)rank * ROWS;
         const bool lin = P.cell == CELL_LINEAR;
         const int bn = (fixed || lin) ? 0 : tl.n * U;
         const int bg = (lin ? tl.n * 4 : 0) + (int)rank * C::GATES;
@@ -263,7 +254,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                 // the segment's producer cell (Table 4 dependence vectors): one acquire of its
                 // (cell, m-block) counter before the segment's first activation load, so inputs
                 // that are ready (x, the layer below) stream in while a later producer finishes
-                if (kc == 0 && sg.scell >= 0 && mine && !FT_DEV_BIT(P.debug, 1)) {
+                if (kc == 0 && sg.scell >= 0 && !FT_DEV_BIT(P.debug, 1)) {
                     FT_TR_BEGIN();
                     wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
                     FT_TR_END(TR_P_FLAG);
@@ -297,12 +288,10 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                     tma_load_4d_hint_addr<CG>(sB0 + (uint32_t)(stage * C::B_BYTES), bm, bar, bn,
                                               fixed ? 0 : sg.krow0 + kc * BK, bg, fixed ? 0 : sg.slice, wpol);
                 }
-            } else if (P.cpair && (!mine || sg.src == SRC_NONE)) {
-                tma_load_2d_hint_addr<CG>(sA0 + (uint32_t)(stage * C::A_BYTES), &M.h, bar, 0, P.zrow, pol_act);
             } else {
                 load_a<CG>(P, M, sA0 + (uint32_t)(stage * C::A_BYTES), bar, sg, kc, arow0, fixed, pol_act);
             }
-            if (++kc == kchunks) { kc = 0; si = P.cpair ? si + 1 : next_segment(seg, si); }
+            if (++kc == kchunks) { kc = 0; si = next_segment(seg, si); }
             if (++stage == C::STAGES) {
                 stage = 0;
                 phase ^= 1;
@@ -336,7 +325,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
     long long tile;
     while (walk_next(P, walk, tl, tile)) {
         Segment seg[3];
-        const int nchunks = (P.cpair ? 3 : segments(P, tl, seg)) * kchunks;
+        const int nchunks = segments(P, tl, seg) * kchunks;
         FT_TR_DECL;
         FT_TR_BEGIN();
         mbar_wait_warp(&tempty[acc], acc_phase ^ 1);
@@ -534,17 +523,11 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     TileId tl;
     long long tile;
     while (walk_next(P, walk, tl, tile)) {
-        TileId tm = tl;  // this CTA's cell (P.cpair: rank 1 takes the pair's second cell)
-        bool mine = true;
-        if (P.cpair && rank == 1) {
-            tm.cell = tl.cell2;
-            mine = tl.has2 != 0;
-        }
-        const Cell c = tm.cell;
+        const Cell c = tl.cell;
         int ci = 0, cj = 0;
-        const long long cprod = mine ? c_producer(P, tm, &ci, &cj) : -1;
-        const int b = P.cpair ? row : tl.m * ROWS * CG + (int)rank * ROWS + row;
-        const bool valid = mine && b < P.B;
+        const long long cprod = c_producer(P, tl, &ci, &cj);
+        const int b = tl.m * ROWS * CG + (int)rank * ROWS + row;
+        const bool valid = b < P.B;
         const int n0 = tl.n * U + half * EPI_UNITS;
         FT_TR_DECL;
         // (0) this tile's bias [4 gates][64 units] → shared memory while the MMAs still run (the
@@ -717,7 +700,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                 const uint32_t h = (uint32_t)(tile * 2654435761u) ^ (uint32_t)(blockIdx.x * 40503u + warp * 977u);
                 __nanosleep(200 + (h & 4095u));
             }
-            if (mine) red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
+            red_release_gpu_add(T.flags + cell_lin(P, c.d, c.i, c.j) * P.MB + tl.m, 1);
         }
         if (leader_thread) {
             FT_TR_END(TR_E_WORK);
@@ -739,7 +722,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
                                       __float_as_uint(cst[4 * v + 2]), __float_as_uint(cst[4 * v + 3])),
                            pol_state);
         }
-        if (split && mine) {
+        if (split) {
             __syncwarp();
             if (lane == 0)
                 red_release_gpu_add(T.flags + cflag_index(P, cell_lin(P, c.d, c.i, c.j), tl.m), 1);
@@ -995,7 +978,7 @@ int choose_band(const Problem& p, int workers) {
 // a hit returns exactly what a fresh encode would.
 struct MapsKey {
     const void *x, *ys, *W, *U, *hb, *xb, *yb;
-    int kind, cell, B, L0, L1, H, D, MB, BM, x_direct, cg, units, dev, cpair;
+    int kind, cell, B, L0, L1, H, D, MB, BM, x_direct, cg, units, dev;
     bool operator==(const MapsKey& o) const { return std::memcmp(this, &o, sizeof(MapsKey)) == 0; }
 };
 struct MapsCache {
@@ -1056,9 +1039,7 @@ cudaError_t encode_maps(const Problem& p, const Tensors& t, EncodeTiledFn enc, b
     if (!encode_blocked(enc, &M.ys, p.kind == KIND_GRID ? t.yb : t.xb,
                         (long long)(p.kind == KIND_GRID ? p.L1 : p.L0) * (p.H / 64) * Bp, err))
         return cudaErrorInvalidValue;
-    // (grid nests: the all-zero K-chunk block of the cell-pair tiles follows the SSA rows)
-    if (!encode_blocked(enc, &M.h, t.hb, hb_rows_total(p) + (p.kind == KIND_GRID ? (long long)p.MB * p.BM : 0), err))
-        return cudaErrorInvalidValue;
+    if (!encode_blocked(enc, &M.h, t.hb, hb_rows_total(p), err)) return cudaErrorInvalidValue;
     if (p.cell == CELL_LINEAR) {
         // W [D][H][H] as (64 n_lo, k, H/64 n_hi, d): a box of 4 (or 2) 64-unit atoms is the
         // 256-unit N tile of one 64-deep K chunk — the same SMEM layout as the LSTM gate atoms
@@ -1149,20 +1130,10 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
     // (profiles/r2_ab_l2_persist.jsonl).  ft_set_l2_persist() sizes or disables it.
     Problem q = p;
     q.persist_layers = 0;
-    // every epilogue warp of every CTA of a tile releases once (cell pairs: only the cell's CTA)
-    q.flag_mult = p.cpair ? EPI_WARPS : CG * EPI_WARPS;
+    q.flag_mult = CG * EPI_WARPS;  // every epilogue warp of every CTA of a tile releases once
     q.x_direct = x_direct;
     q.band = choose_band(p, (int)(grid / CG));
     if (q.hring) hb_layout(q, q.band);
-    if (q.cpair) {  // cell-pair tiles (grid): tiles per the pairing of this order; per-cell counters
-        q.ntiles = count_pairs(q) * q.naxes * q.NT;  // complete at NT·naxes·EPI_WARPS (one CTA per cell)
-        q.zrow = (int)hb_rows_total(q);
-        e = cudaMemsetAsync(static_cast<uint8_t*>(t.hb) + (size_t)q.zrow * 128, 0, (size_t)p.MB * p.BM * 128, s);
-        if (e != cudaSuccess) {
-            if (err) *err = std::string("zero block: ") + cudaGetErrorString(e);
-            return e;
-        }
-    }
     // Dedicated owners for layer 0 of a dilated nest (TileWalk owner mode 2): layer 0 has
     // dilation 1, the only recurrence without slack, so its slabs get their own CTA pairs (cell
     // state in registers, no queueing behind other layers' tiles); the other layers run
@@ -1237,7 +1208,6 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
                         "> grid=" + std::to_string(grid) + " cluster=" + std::to_string(CG) +
                         " cooperative=" + std::to_string(coop) + " band=" + std::to_string(q.band) +
                         " skew=" + std::to_string(seq_skew(q)) + " owner=" + std::to_string(q.owner) +
-                        " cell_pairs=" + std::to_string(q.cpair) +
                         " x_direct=" + std::to_string(q.x_direct) + " persist_layers=" +
                         std::to_string(q.persist_layers) + " resident_layers=" +
                         std::to_string(q.resident_layers) + " stress=" + std::to_string((q.debug & 64) != 0));
@@ -1262,7 +1232,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     MapsKey key;
     std::memset(&key, 0, sizeof(key));
     key = MapsKey{t.x, t.ys, t.W, t.U, t.hb, t.xb, t.yb, p.kind, p.cell, p.B, p.L0, p.L1, p.H, p.D,
-                  p.MB, p.BM, (int)x_direct, CG, U, dev, p.cpair};
+                  p.MB, p.BM, (int)x_direct, CG, U, dev};
     Maps M;
     if (!maps_cache().find(key, &M)) {
         const cudaError_t ee = encode_maps<CG, U>(p, t, enc, x_direct, &M, err);
@@ -1343,17 +1313,7 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
     // N-tile width: 64 units by default; 32 units only when a diagonal at 64 units would give
     // under a quarter of the CTA groups a tile: twice the tiles, half the per-tile latency on the
     // dependency chain, but 1.5x the operand traffic per FLOP.
-    int cg = p.BM == 2 * ROWS ? 2 : 1;
-    // grid nests with one 128-row m-block: cell pairs on CTA pairs (one weight tile per two
-    // cells of a diagonal group).  FT_GRID_PAIRS=0 keeps one cell per CTA.
-    Problem pp = p;
-    if (cg == 1 && p.kind == KIND_GRID && p.cell == CELL_LSTM && p.MB == 1) {
-        const char* e = getenv("FT_GRID_PAIRS");
-        if (!(e && e[0] == '0')) {
-            pp.cpair = 1;
-            cg = 2;
-        }
-    }
+    const int cg = p.BM == 2 * ROWS ? 2 : 1;
     int dev = 0, nsm = 148;
     if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     long long max_cells = 0;
@@ -1375,9 +1335,8 @@ cudaError_t launch_wavefront_bf16(const Problem& p, const Tensors& t, cudaStream
     //  32-unit split now only pays on diagonals a quarter of that wide)
     int units = (4 * max_cells * p.naxes * p.MB * p.NT < nsm / cg && p.cell == CELL_LSTM && p.H % 32 == 0) ? 32 : 64;
     if (const char* env = getenv("FT_TILE_UNITS")) units = atoi(env) == 32 && p.cell == CELL_LSTM ? 32 : 64;
-    if (pp.cpair) units = 64;
     if (units == 64)
-        return cg == 2 ? launch_cg<2, 64>(pp, t, s, err) : launch_cg<1, 64>(p, t, s, err);
+        return cg == 2 ? launch_cg<2, 64>(p, t, s, err) : launch_cg<1, 64>(p, t, s, err);
     Problem q = p;
     q.BNU = 32;
     q.NT = p.H / 32;
