@@ -67,5 +67,15 @@ ft.check(ft.ft_stacked_lstm_fwd_hostio(B, T, H, D, ft.FT_BF16, x_h.data_ptr(), W
                                        ws.data_ptr(), nb, s.cuda_stream))
 s.synchronize()
 os.environ.pop("FT_BAND")
+# round 2 (this round) features
+os.environ["FT_CLUSTER"] = "1"                            # cluster kernel, 16-unit slices (H = 128)
+os.environ["FT_CLUSTER_UNITS"] = "16"
+run_seq(40, 6, 128, 3, torch.bfloat16)
+os.environ.pop("FT_CLUSTER_UNITS")
+os.environ.pop("FT_CLUSTER")
+os.environ["FT_BAND"] = "2"                               # SSA slot rings wrapping under bands
+run_seq(256, 11, 64, 6, torch.bfloat16, resident="0")
+os.environ.pop("FT_BAND")
+run_seq(256, 11, 64, 4, torch.bfloat16, dil=[1, 2, 4, 3], resident="0")  # rings + layer-0 owners (default)
 torch.cuda.synchronize()
 print("sanitize cases done")
