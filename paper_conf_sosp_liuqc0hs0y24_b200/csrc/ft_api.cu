@@ -102,7 +102,7 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         // a6 for the bf16 streaming kernel: the SSA buffer hb as per-layer rings (ft_common.cuh
         // hb_slot_row) plus two T-step regions for band-boundary layers — C3: 1600 rows of
         // (d, t) → 16·4 + 200.  The launcher lays the slots out once the band is known.
-        if (dt == FT_BF16 && cell == ft::CELL_LSTM && ft::hb_ring_eligible(*p)) {
+        if (dt == FT_BF16 && cell == ft::CELL_LSTM && ft::hb_ring_eligible(*p) && !ft::env_off("FT_SSA_RING")) {
             long long rows = 2ll * L0;
             for (int d = 0; d < D; ++d) rows += ft::hb_ring_len(dil[d], L0);
             if (rows < (long long)D * L0) {

@@ -14,6 +14,10 @@ namespace ft {
 // Environment knobs (every one is documented in include/ft.h; none changes a result beyond the
 // summation-order freedom that header states).  Read per call, so a test can flip them.
 inline const char* env_str(const char* name) { return getenv(name); }
+inline bool env_off(const char* name) {  // set to "0"
+    const char* e = getenv(name);
+    return e && e[0] == '0' && e[1] == 0;
+}
 inline bool env_flag(const char* name) {  // set and not "0"
     const char* e = getenv(name);
     return e && e[0] && !(e[0] == '0' && e[1] == 0);
