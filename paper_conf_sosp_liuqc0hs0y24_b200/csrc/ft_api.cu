@@ -290,7 +290,7 @@ void set_last_error(const std::string& msg) { g_last_error = msg; }
 void set_last_launch(const std::string& s) { g_last_launch = s; }
 long long c_ring_elems(const Problem& p) {
     if (p.kind == KIND_SEQ) return (long long)p.ring_off[p.D] * c_slot_elems(p);
-    return ((long long)p.D * 2 * p.L1 + (long long)p.D * p.L0 * 2) * c_slot_elems(p);
+    return ((long long)p.D * p.L1 + (long long)p.D * p.L0) * c_slot_elems(p);
 }
 }  // namespace ft
 

@@ -524,8 +524,11 @@ FT_HD int src_rows(const Problem& p, int src) {
 // Cell-state ring (fp32).  KIND_SEQ: layer d owns ring_len_d = min(T, 2·s_d) slots
 // [ring_off[d], ring_off[d+1]); slot of step t is t mod ring_len_d.  The slot written by
 // (d, t) last held c(d, t - 2s_d), read by (d, t - s_d) — a direct producer of (d, t), so the
-// reuse is ordered by the flag protocol.  KIND_GRID: c^x ring of 2 slots over i
-// ([D][2][Ly] slots) and c^y ring of 2 slots over j ([D][Lx][2] slots), same argument.
+// reuse is ordered by the flag protocol.  KIND_GRID: ONE c^x slot per (depth, column j) and one
+// c^y slot per (depth, row i) ([D][Ly] + [D][Lx] slots): c^x(d, i−1, j) is read only by cell
+// (d, i, j) — the same threads that then overwrite the same elements with c^x(d, i, j) — and the
+// next writer (d, i+1, j) depends on (d, i, j) (e_x of Table 4), so one slot carries the chain.
+// (Round 1 kept 2 slots: 32 MiB of rings per C5 depth instead of 16.)
 // Inside a slot the layout is [H/4][B][4]: 4 units of one batch row are one 16-byte vector and
 // consecutive batch rows are adjacent, so an epilogue warp (one thread per batch row) loads and
 // stores whole 512-byte runs.  (A [B][H] slot made every warp store 32 partial sectors 4 KiB
@@ -539,9 +542,9 @@ FT_HD long long c_ring_index(const Problem& p, int d, int i, int j, int a, int b
         const int len = p.ring_off[d + 1] - p.ring_off[d];
         return c_slot_index(p, p.ring_off[d] + i % len, b, n);
     }
-    if (a == 0) return c_slot_index(p, ((long long)d * 2 + (i & 1)) * p.L1 + j, b, n);
-    const long long base = (long long)p.D * 2 * p.L1;
-    return c_slot_index(p, base + ((long long)d * p.L0 + i) * 2 + (j & 1), b, n);
+    if (a == 0) return c_slot_index(p, (long long)d * p.L1 + j, b, n);
+    const long long base = (long long)p.D * p.L1;
+    return c_slot_index(p, base + (long long)d * p.L0 + i, b, n);
 }
 
 // The cell whose c the tile's epilogue reads (its c-producer), or -1 (zero initial state).

@@ -949,18 +949,21 @@ int choose_band(const Problem& p, int workers) {
         return b > 0 && b < p.D ? b : 0;
     }
     if (p.kind == KIND_GRID) {
-        // grid nests carry two fp32 cell states per cell (c^x, c^y); their rings for all depths
-        // are D · 2 · (Lx + Ly) slots of B·H fp32.  A depth band's live L2 set is its rings plus
-        // its weights (2 axes x 4 gates x H x 3H bf16 per depth); when the whole nest's set exceeds
-        // a 64 MiB L2 budget (C5: 128 MiB of rings + 48 MiB of weights), run depth bands whose set
-        // fits.  C5: band 1 (32 + 12 MiB).  Same box: DRAM 9.6 GB (paper order) -> 5.9 GB (bands
-        // of 2) -> 2.95 GB (bands of 1) per forward at the same time (5.94 / 5.95 ms,
-        // profiles/r2_ab_grid_bands.txt, profiles/rnd2_ab_c5_band1.txt)
-        const double ring_per_depth = 2.0 * (p.L0 + p.L1) * (double)p.B * p.H * 4.0;
+        // grid nests carry two fp32 cell states per cell (c^x, c^y): one slot per column / row
+        // and depth, (Lx + Ly) slots of B·H fp32 per depth.  A depth band's live L2 set is its
+        // rings, its weights (2 axes x 4 gates x H x 3H bf16 per depth) and the SSA rows it
+        // streams; when the whole nest's set exceeds the budget, run depth bands whose rings and
+        // weights fit in 40 MiB.  C5: 16 + 12 MiB per depth -> bands of 1.  Same box: DRAM 9.6 GB
+        // (paper order, 2-slot rings) -> 5.9 GB (bands of 2) -> 2.95 GB (bands of 1) -> 2.33 GB
+        // (bands of 1, 1-slot rings) per forward, time unchanged; bands of 2 with 1-slot rings
+        // spill again (4.5 GB) at the same time (profiles/r2_ab_grid_bands.txt,
+        // profiles/rnd2_ab_c5_band1.txt, profiles/rnd2_ab_c5_cring.txt)
+        const double ring_per_depth = (double)(p.L0 + p.L1) * (double)p.B * p.H * 4.0;
         const double w_per_depth = 2.0 * 4.0 * p.H * 3.0 * p.H * 2.0;
         const double per_depth = ring_per_depth + w_per_depth;
-        if (per_depth * p.D <= 64.0 * 1024 * 1024) return 0;
-        const int band = (int)((64.0 * 1024 * 1024) / per_depth);
+        const double budget = 40.0 * 1024 * 1024;
+        if (per_depth * p.D <= budget) return 0;
+        const int band = (int)(budget / per_depth);
         return band < 1 ? 1 : (band >= p.D ? 0 : band);
     }
     if (p.kind != KIND_SEQ) return 0;
