@@ -95,7 +95,7 @@ ft_status make_problem(int kind, int B, int L0, int L1, int H, int D, const int*
         for (int d = 0; d < D; ++d) {
             p->dil[d] = dil[d];
             p->ring_off[d] = off;
-            const long long len = 2ll * dil[d] < L0 ? 2ll * dil[d] : L0;
+            const long long len = dil[d] < L0 ? dil[d] : L0;  // one slot per residue of t mod s_d
             off += (int)len;
         }
         p->ring_off[D] = off;

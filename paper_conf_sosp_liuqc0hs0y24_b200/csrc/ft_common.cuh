@@ -521,10 +521,11 @@ FT_HD int src_rows(const Problem& p, int src) {
     return src == SRC_X ? p.L0 : (src == SRC_YS ? p.L1 : h_rows(p));
 }
 
-// Cell-state ring (fp32).  KIND_SEQ: layer d owns ring_len_d = min(T, 2·s_d) slots
-// [ring_off[d], ring_off[d+1]); slot of step t is t mod ring_len_d.  The slot written by
-// (d, t) last held c(d, t - 2s_d), read by (d, t - s_d) — a direct producer of (d, t), so the
-// reuse is ordered by the flag protocol.  KIND_GRID: ONE c^x slot per (depth, column j) and one
+// Cell-state ring (fp32).  KIND_SEQ: layer d owns ring_len_d = min(T, s_d) slots
+// [ring_off[d], ring_off[d+1]); slot of step t is t mod ring_len_d.  The slot cell (d, t) writes
+// held c(d, t - s_d), which only (d, t) itself reads — the same threads, the same elements, read
+// before they are overwritten — and the next writer (d, t + s_d) depends on (d, t), so the reuse
+// is ordered by the flag protocol.  (Round 1 kept 2·s_d slots per layer.)  KIND_GRID: ONE c^x slot per (depth, column j) and one
 // c^y slot per (depth, row i) ([D][Ly] + [D][Lx] slots): c^x(d, i−1, j) is read only by cell
 // (d, i, j) — the same threads that then overwrite the same elements with c^x(d, i, j) — and the
 // next writer (d, i+1, j) depends on (d, i, j) (e_x of Table 4), so one slot carries the chain.
