@@ -57,7 +57,7 @@ parts = {"sync": E5[t] - R[t - 1], "issue": E2[t] - E5[t], "land": E7[t] - E2[t]
          "tail": E3[t] - E7[t], "epi": R[t] - E3[t], "step": R[t] - R[t - 1]}
 print(f"B={B} T={T} H={H} U={U}: " + "  ".join(f"{k} {np.median(v):.2f}" for k, v in parts.items()) + " us")
 # every event of step t+1 relative to R(t) (the release that enables it)
-rel = {f"E{k}": np.median(ev[t, :, k].max(1) - R[t - 1]) for k in range(13)}
-rel_min = {f"E{k}": np.median(ev[t, :, k].min(1) - R[t - 1]) for k in range(13)}
+rel = {f"E{k}": np.median(ev[t, :, k].max(1) - R[t - 1]) for k in range(16)}
+rel_min = {f"E{k}": np.median(ev[t, :, k].min(1) - R[t - 1]) for k in range(16)}
 print("  rel to R(t-1) max over tiles: " + " ".join(f"{k}={v:.2f}" for k, v in rel.items()))
 print("  rel to R(t-1) min over tiles: " + " ".join(f"{k}={v:.2f}" for k, v in rel_min.items()))

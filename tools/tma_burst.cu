@@ -56,7 +56,37 @@ __global__ void __launch_bounds__(256, 1) burst(const __grid_constant__ CUtensor
             }
         }
         if (mode == 4) asm volatile("barrier.cluster.arrive.release.aligned; barrier.cluster.wait.acquire.aligned;" ::: "memory");
-        if (threadIdx.x == 0) {
+        if (mode == 5 && threadIdx.x < 32) {  // every lane k < nload issues load k (one warp-wide TMA instruction)
+            __syncwarp();
+            const int k = threadIdx.x;
+            const uint64_t t_seen = gtime_seen;
+            if (k < nload) {
+                const int src = (cta + k) % ncta;
+                const uint32_t bar = su32(&bars[k]);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(CHUNK) : "memory");
+                const int row = ((r & 1) * ncta + src) * 128;
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];"
+                    ::"r"(su32(smem + k * CHUNK)), "l"(&map), "r"(0), "r"(row), "r"(bar) : "memory");
+            }
+            const uint64_t t_i = gtime();
+            __syncwarp();
+            if (k == 0) {
+                uint64_t t_land[MAXL];
+                for (int j = 0; j < nload; ++j) {
+                    const uint32_t bar = su32(&bars[j]);
+                    uint32_t ok = 0;
+                    while (!ok)
+                        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                                     : "=r"(ok) : "r"(bar), "r"((uint32_t)(r & 1)) : "memory");
+                    t_land[j] = gtime();
+                }
+                unsigned long long* o = out + ((size_t)r * ncta + cta) * (1 + 2 * MAXL);
+                o[0] = t_seen;
+                for (int j = 0; j < nload; ++j) { o[1 + j] = t_i; o[1 + MAXL + j] = t_land[j]; }
+            }
+        }
+        if (threadIdx.x == 0 && mode != 5) {
             const uint64_t t_seen = gtime_seen;
             uint64_t t_iss[MAXL];
             for (int k = 0; k < nload; ++k) {
@@ -139,9 +169,9 @@ int main(int argc, char** argv) {
         }
         const int smem = MAXL * CHUNK + 1024;
         CK(cudaFuncSetAttribute(burst, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-        const char* names[] = {"others", "same", "hint", "2cta", "mcast8"};
-        for (int mode = 0; mode < 5; ++mode)
-            for (int nload : {8}) {
+        const char* names[] = {"others", "same", "hint", "2cta", "mcast8", "lanes"};
+        for (int mode : {0, 1, 5})
+            for (int nload : {1, 8, 12}) {
                 CK(cudaMemset(flags, 0, ROUNDS * sizeof(int)));
                 cudaLaunchConfig_t cfg = {};
                 cfg.gridDim = dim3(ncta);
