@@ -44,6 +44,15 @@ namespace ft {
 __device__ unsigned long long g_cev[4096 * 8];
 __device__ int g_cev_cta = 0;
 #define FT_CEV(t, k) do { if (blockIdx.x == g_cev_cta && (t) < 4096) g_cev[(t) * 8 + (k)] = globaltimer_ns(); } while (0)
+// per layer: %globaltimer when slice 0's epilogue saw the accumulator of step t (all layers, one run)
+__device__ unsigned long long g_lev[64 * 1024];
+#define FT_LEV(d, t) do { if ((d) < 64 && (t) < 1024) g_lev[(d) * 1024 + (t)] = globaltimer_ns(); } while (0)
+extern "C" __attribute__((visibility("default"))) int ft_debug_cluster_layer_events(unsigned long long* host, int D, int T) {
+    cudaDeviceSynchronize();
+    for (int d = 0; d < D && d < 64; ++d)
+        if (cudaMemcpyFromSymbol(host + (size_t)d * T, g_lev, (size_t)T * 8, (size_t)d * 1024 * 8) != cudaSuccess) return -1;
+    return D;
+}
 extern "C" __attribute__((visibility("default"))) int ft_debug_cluster_events(unsigned long long* host, int nsteps, int cta) {
     if (nsteps > 4096) nsteps = 4096;
     cudaDeviceSynchronize();
@@ -53,6 +62,7 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_cluster_events(un
 }
 #else
 #define FT_CEV(t, k) ((void)0)
+#define FT_LEV(d, t) ((void)0)
 #endif
 
 namespace {
@@ -296,6 +306,7 @@ wavefront_cluster_kernel(const __grid_constant__ Problem P, const __grid_constan
         for (int t = 0; t < P.L0; ++t) {
             mbar_wait(&tfull[acc], acc_phase);
             if (sender) FT_CEV(t, 2);
+            if (sender && j == 0) FT_LEV(d, t);
             tc_fence_after();
             const uint32_t tbase = tmem_base + (uint32_t)(acc * KN) + ((uint32_t)(q * 32) << 16) + half * KEU;
             uint32_t hp[KEU / 2];

@@ -407,13 +407,15 @@ def test_bf16_stress_delayed_release(B, T, H, D, dil, monkeypatch):
     _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx="stress")
 
 
-@pytest.mark.parametrize("band", ["0", "2"])
-def test_bf16_cuda_graph_capture_replay(band, monkeypatch):
+@pytest.mark.parametrize("band,shape", [("0", (130, 5, 128, 3)), ("2", (130, 5, 128, 3)),
+                                        ("0", (64, 9, 256, 8))])
+def test_bf16_cuda_graph_capture_replay(band, shape, monkeypatch):
     """The forward (counter reset + input pack + persistent kernel) captures into a CUDA graph
     and replays with new inputs copied into the captured buffers (the serving path) — in the
-    paper order and in layer bands with the owner-computes walk (C3's schedule)."""
+    paper order, in layer bands with the owner-computes walk (C3's schedule), and through the
+    DSMEM cluster kernel (C2's; a replay removes the call's host latency)."""
     monkeypatch.setenv("FT_BAND", band)
-    B, T, H, D = 130, 5, 128, 3
+    B, T, H, D = shape
     p1 = ftgen.stacked_inputs(B, T, H, D, 1818, "bf16")
     p2 = ftgen.stacked_inputs(B, T, H, D, 1819, "bf16")
     x, W, U = (dev(p1[k], torch.bfloat16) for k in ("x", "W", "U"))
@@ -429,6 +431,8 @@ def test_bf16_cuda_graph_capture_replay(band, monkeypatch):
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g, stream=s):
         ft.stacked_lstm(x, W, U, b, workspace=ws, out=out, stream=s)
+    if H == 256:
+        assert "wavefront_cluster_kernel" in ft.ft_last_launch(), ft.ft_last_launch()
     x.copy_(dev(p2["x"], torch.bfloat16))
     g.replay()
     torch.cuda.synchronize()
