@@ -63,6 +63,8 @@ struct Problem {
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
+    int rec_first;       // KIND_SEQ: a layer with dilation >= 2 runs its K loop recurrent half
+                         // first (see segments)
     int hring;           // bf16 streaming KIND_SEQ: hb holds a ring of slots per layer instead of
                          // every (d, t) row (see hb_slot_row); 0 = one row per (d, t)
     int hb_rows;         // hring: rows of hb the workspace reserves (Σ ring lengths + 2·L0)
@@ -494,6 +496,16 @@ FT_HD int segments(const Problem& p, const TileId& tl, Segment seg[3]) {
         seg[1] = Segment{rec ? SRC_H : SRC_NONE, rec ? hb_slot_row(p, c.d, c.i - s, 0, 0) : 0,
                          W_REC, c.d, 0, rec ? (int)cell_lin(p, c.d, c.i - s, 0) : -1, 0};
         seg[2] = Segment{SRC_NONE, 0, W_REC, c.d, 0, -1, 0};
+        // Dilation s >= 2: the recurrent producer (d, t − s) lies s − 1 diagonals before the
+        // depth producer (d − 1, t), so it is (almost always) ready first.  Running its half of
+        // the K loop first leaves only the depth half behind the depth edge, which cuts the
+        // latency of every layer-to-layer hop of a dilated nest by one half-K of MMAs.  The sum
+        // is the same (the K halves are added in a different order: equal within rounding).
+        if (p.rec_first && rec && s >= 2 && c.d > 0) {
+            const Segment t0 = seg[0];
+            seg[0] = seg[1];
+            seg[1] = t0;
+        }
     } else {
         const int a = tl.axis, sl = c.d * 2 + a;
         if (c.d == 0)

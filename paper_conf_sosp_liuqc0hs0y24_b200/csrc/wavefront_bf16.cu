@@ -1152,6 +1152,11 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
             p.naxes == 1 && p.D >= 2 && p.dil[0] == 1 && 2ll * p.NT <= grid / CG)
             q.owner = 2;
     }
+    // recurrent half first for dilated layers (segments); FT_REC_FIRST=0 keeps the input half first
+    {
+        const char* e = getenv("FT_REC_FIRST");
+        q.rec_first = !(e && e[0] == '0');
+    }
 #ifdef FT_DEV_EXPERIMENTS
     if (const char* e = getenv("FT_L2POL")) q.l2pol = atoi(e);  // L2 policy experiments (dev builds)
 #endif
