@@ -791,7 +791,8 @@ FT_API long long ft_tile_walk(int depth, int seq, int band, int skew, int owner,
     p.skew = skew;
     p.owner = (owner == 1 && band > 0 && band < depth && ft::seq_band(p) * ntiles_n <= nworkers)
                   ? 1
-                  : (owner == 2 && 2 * ntiles_n <= nworkers ? 2 : 0);
+                  : (owner == 2 && 2 * ntiles_n <= nworkers ? 2
+                                                             : (owner == 3 && depth * ntiles_n <= nworkers ? 3 : 0));
     for (int d = 0; d < depth; ++d) p.dil[d] = 1;
     ft::TileWalk w = ft::walk_begin(p, worker, nworkers);
     ft::TileId tl;

@@ -286,6 +286,12 @@ FT_HD TileId decode_tile(const Problem& p, Cursor& cur, long long tile) {
 //    worker's own previous tile, so co-resident workers cannot deadlock.
 // `tid` identifies the tile for tracing: the global sequence index (round-robin) or
 // cell_lin·NT + n (owner).
+//  * every layer owned (p.owner == 3, dilated nests with D·NT <= workers): worker w owns
+//    (layer w / NT, N-tile w % NT) for t = 0 .. T−1.  Layer e's tile t needs (e − 1, t) of
+//    another worker and (e, t − s_e) of its own earlier tiles, and layer 0 depends only on its own
+//    steps, so the waits form no cycle.  Each layer then advances at the pace of the layer below
+//    with a constant lag instead of queueing behind other layers' tiles.  The cell state stays
+//    in registers for layers of dilation 1; the others keep the c ring.
 //  * layer-0 owners (p.owner == 2, dilated nests whose layer 0 has dilation 1: its T-step
 //    recurrence is the only chain without slack): worker w < NT owns (layer 0, N-tile w) for
 //    t = 0 .. T−1, with its cell state in registers; the other workers take the remaining
@@ -315,6 +321,11 @@ FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
     if (p.owner == 1 && worker < seq_band(p) * p.NT) {
         w.e = worker / p.NT;
         w.n = worker - w.e * p.NT;
+    } else if (p.owner == 3) {
+        if (worker < p.D * p.NT) {
+            w.e = worker / p.NT;
+            w.n = worker - w.e * p.NT;
+        }
     } else if (p.owner == 2) {
         if (worker < p.NT) {
             w.e = 0;
@@ -334,6 +345,16 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
         tl = decode_tile(p, w.cur, w.tile);
         tid = w.tile;
         w.tile += w.stride;
+        return true;
+    }
+    if (p.owner == 3) {  // every layer owned: worker (layer e, N-tile n) runs t = 0 .. T-1
+        if (w.e < 0 || w.t >= p.L0) return false;
+        tl.cell = Cell{w.e + w.t, w.e, w.t, 0, 0, w.e + w.t};
+        tl.axis = 0;
+        tl.m = 0;
+        tl.n = w.n;
+        tid = cell_lin(p, w.e, w.t, 0) * p.NT + w.n;
+        ++w.t;
         return true;
     }
     if (p.owner == 2 && w.e == -2) {  // round-robin over the tiles of layers >= 1

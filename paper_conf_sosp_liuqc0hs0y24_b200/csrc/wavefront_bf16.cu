@@ -513,7 +513,9 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     // owner-computes (TileWalk): this thread's rows x units of the slab are the same in every
     // tile, so the cell state stays in registers (cst) from step t to t + 1 — no c ring, no
     // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
-    const bool own = P.owner == 1 || (P.owner == 2 && (int)(blockIdx.x / CG) < P.NT);
+    const int worker = (int)(blockIdx.x / CG);
+    const bool own = P.owner == 1 || (P.owner == 2 && worker < P.NT) ||
+                     (P.owner == 3 && worker < P.D * P.NT && P.dil[worker / P.NT] == 1);
     const bool split = P.band > 0 && !own;
     float cst[EPI_UNITS];
 #pragma unroll
@@ -1151,6 +1153,12 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
         if (want && q.band == 0 && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.MB == 1 &&
             p.naxes == 1 && p.D >= 2 && p.dil[0] == 1 && 2ll * p.NT <= grid / CG)
             q.owner = 2;
+        // every layer owned (TileWalk mode 3) when all D·NT slabs get a pair: each layer then
+        // advances at the pace of the layer below with a constant lag instead of queueing behind
+        // other layers' tiles (C4 0.750 -> 0.737 ms pipelined same-box,
+        // profiles/rnd2_ab_owner_all.txt); FT_OWNER_ALL=0 keeps mode 2
+        const char* ea = getenv("FT_OWNER_ALL");
+        if (q.owner == 2 && !(ea && ea[0] == '0') && (long long)p.D * p.NT <= grid / CG) q.owner = 3;
     }
     // recurrent half first for dilated layers (segments); FT_REC_FIRST=0 keeps the input half first
     {

@@ -667,9 +667,30 @@ def test_bf16_layer0_owner_walk(dil, monkeypatch):
     ref_gpu = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
     assert "owner=0" in ft.ft_last_launch()
     monkeypatch.delenv("FT_OWNER_L0")
+    monkeypatch.setenv("FT_OWNER_ALL", "0")
     got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
     assert "owner=2" in ft.ft_last_launch()
     _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"l0 owner {dil}")
+    for k in ALL:
+        assert torch.equal(got[k], ref_gpu[k]), k
+
+
+@pytest.mark.parametrize("dil", [[1, 2, 4, 8, 16, 32], [1, 3, 2], [1, 1, 2, 1]])
+def test_bf16_all_layers_owner_walk(dil, monkeypatch):
+    """Every layer owned (TileWalk mode 3, the default for dilated nests when D·NT slabs fit):
+    parity with the oracle and bitwise equality with the layer-0 owner walk (FT_OWNER_ALL=0: the
+    same tiles and K order, another assignment); dilation-1 layers above layer 0 keep c in
+    registers, the others use the c ring."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    D = len(dil)
+    p = ftgen.stacked_inputs(256, 9, 128, D, 2030 + D, "bf16")
+    monkeypatch.setenv("FT_OWNER_ALL", "0")
+    ref_gpu = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    assert "owner=2" in ft.ft_last_launch()
+    monkeypatch.setenv("FT_OWNER_ALL", "1")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    assert "owner=3" in ft.ft_last_launch()
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True), torch.bfloat16, ALL, ctx=f"all owners {dil}")
     for k in ALL:
         assert torch.equal(got[k], ref_gpu[k]), k
 

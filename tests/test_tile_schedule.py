@@ -277,6 +277,36 @@ def test_layer0_owner_walk(D, T, nt, nw, dil):
             left[(d, t)] -= 1
 
 
+@pytest.mark.parametrize("D,T,nt,nw,dil", [
+    (6, 12, 8, 74, [1, 2, 4, 8, 16, 32]), (3, 7, 4, 13, [1, 3, 2]), (4, 5, 2, 9, [1, 1, 2, 1]),
+])
+def test_all_layers_owner_walk(D, T, nt, nw, dil):
+    """Owner mode 3 (dilated nests, D·nt <= workers): worker w owns (layer w // nt, N-tile
+    w % nt) for t ascending; workers past D·nt are idle.  Coverage and deadlock freedom with the
+    dilated dependences (d-1, t) and (d, t - s_d); too few workers fall back to the round-robin
+    walk."""
+    walks = [ft.ft_tile_walk(D, T, 0, 1, 3, nt, w, nw) for w in range(nw)]
+    allt = sorted(x for w in walks for x in w)
+    assert allt == [(d, t, n) for d in range(D) for t in range(T) for n in range(nt)]
+    for w in range(nw):
+        assert walks[w] == ([(w // nt, t, w % nt) for t in range(T)] if w < D * nt else [])
+    left = {(d, t): nt for d in range(D) for t in range(T)}
+    heads = [0] * nw
+    while any(heads[w] < len(walks[w]) for w in range(nw)):
+        done = []
+        for w in range(nw):
+            if heads[w] < len(walks[w]):
+                d, t, n = walks[w][heads[w]]
+                if (d == 0 or left[(d - 1, t)] == 0) and (t < dil[d] or left[(d, t - dil[d])] == 0):
+                    done.append(w)
+        assert done, "deadlock"
+        for w in done:
+            d, t, n = walks[w][heads[w]]
+            heads[w] += 1
+            left[(d, t)] -= 1
+    assert ft.ft_tile_walk(D, T, 0, 1, 3, nt, 0, D * nt - 1) == ft.ft_tile_walk(D, T, 0, 1, 0, nt, 0, D * nt - 1)
+
+
 @pytest.mark.parametrize("D,Lx,Ly,band", [(4, 3, 4, 1), (4, 5, 2, 2), (5, 4, 4, 3), (3, 1, 6, 1), (2, 6, 1, 1)])
 def test_grid_depth_bands_are_legal(D, Lx, Ly, band):
     """Grid nests in depth bands (band after band, each a wavefront over i + j + (d - d0)): every
