@@ -485,7 +485,7 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
     HostIoStreams hs;
     StreamWaitValue32Fn wait_value = nullptr;
     StreamWriteValue32Fn write_value = nullptr;
-    int per_step = 0, per_chunk = 0;
+    int per_step = 0, per_chunk = 0, per_step0 = 0;
     const int chunk = hostio_chunk(), nchunks = (seq + chunk - 1) / chunk;
     const bool overlap = dt == FT_BF16 && !getenv("FT_HOSTIO_SERIAL") &&
                          ft::bf16_kernel_choice(p) == 2 && hostio_streams(&hs, &wait_value, &write_value);
@@ -494,6 +494,7 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
         t.ychunk = chunk;
         t.ysig_per_step = &per_step;
         t.ysig_per_chunk = &per_chunk;
+        t.nsig0_per_step = &per_step0;
         t.xsig = reinterpret_cast<int*>(ws + hp.xsig_off);
         t.xchunk = chunk;
         t.nsig = reinterpret_cast<int*>(ws + hp.nsig_off);
@@ -541,7 +542,8 @@ FT_API ft_status ft_stacked_lstm_fwd_hostio(int batch, int seq, int hidden, int 
         const size_t hrow = (size_t)hidden * es, crow = (size_t)hidden * 4;
         const size_t hpitch = (size_t)depth * hrow, cpitch = (size_t)depth * crow;
         for (int d = 0; d < depth && se == cudaSuccess; ++d) {
-            if (wait_value(hs.state, (CUdeviceptr)(t.nsig + d), (cuuint32_t)per_step, CU_STREAM_WAIT_VALUE_GEQ) !=
+            const int need = (d == 0 && per_step0 > 0) ? per_step0 : per_step;
+            if (wait_value(hs.state, (CUdeviceptr)(t.nsig + d), (cuuint32_t)need, CU_STREAM_WAIT_VALUE_GEQ) !=
                 CUDA_SUCCESS) {
                 se = cudaErrorUnknown;
                 break;
@@ -792,7 +794,9 @@ FT_API long long ft_tile_walk(int depth, int seq, int band, int skew, int owner,
     p.owner = (owner == 1 && band > 0 && band < depth && ft::seq_band(p) * ntiles_n <= nworkers)
                   ? 1
                   : (owner == 2 && 2 * ntiles_n <= nworkers ? 2
-                                                             : (owner == 3 && depth * ntiles_n <= nworkers ? 3 : 0));
+                     : (owner == 3 && depth * ntiles_n <= nworkers ? 3
+                     : (owner == 4 && (depth + 1) * ntiles_n <= nworkers ? 3 : 0)));
+    if (owner == 4 && p.owner == 3) p.nt0 = 2 * ntiles_n;
     for (int d = 0; d < depth; ++d) p.dil[d] = 1;
     ft::TileWalk w = ft::walk_begin(p, worker, nworkers);
     ft::TileId tl;

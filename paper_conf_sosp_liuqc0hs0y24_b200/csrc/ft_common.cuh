@@ -63,6 +63,8 @@ struct Problem {
     int band, skew;      // KIND_SEQ order (0 = defaults D, 1): layers are processed in bands of
                          // `band` consecutive layers, each band a wavefront π = t + skew·(d − d0)
                          // (see next_cell); bands run one after the other
+    int nt0;             // owner mode 3: layer 0's N-tiles when layer 0 runs narrower slabs than
+                         // the other layers (0 = NT, the same width)
     int rec_first;       // KIND_SEQ: a layer with dilation >= 2 runs its K loop recurrent half
                          // first (see segments)
     int hring;           // bf16 streaming KIND_SEQ: hb holds a ring of slots per layer instead of
@@ -216,6 +218,12 @@ FT_HD int tiles_per_cell(const Problem& p) { return p.naxes * p.MB * p.NT; }
 // Flags: one int per (cell, m-block); complete when it reaches naxes * NT * flag_mult
 // (cell-granular protocol of the fp32 kernel).
 FT_HD int flag_target(const Problem& p) { return p.naxes * p.NT * p.flag_mult; }
+// N-tiles of layer 0 (owner mode 3 may run layer 0 in narrower slabs) and the readiness target
+// of a cell of layer d (every epilogue warp of every tile of the cell releases once)
+FT_HD int nt_layer0(const Problem& p) { return p.nt0 > 0 ? p.nt0 : p.NT; }
+FT_HD int flag_target_layer(const Problem& p, int d) {
+    return d == 0 ? p.naxes * nt_layer0(p) * p.flag_mult : flag_target(p);
+}
 
 // Under layer bands the bf16 streaming kernel publishes a cell twice: the h-ready counter
 // flags + cell·MB + m (what the next cells' MMAs read: released as soon as h is stored) and the
@@ -322,9 +330,13 @@ FT_HD TileWalk walk_begin(const Problem& p, int worker, int nworkers) {
         w.e = worker / p.NT;
         w.n = worker - w.e * p.NT;
     } else if (p.owner == 3) {
-        if (worker < p.D * p.NT) {
-            w.e = worker / p.NT;
-            w.n = worker - w.e * p.NT;
+        const int nt0 = nt_layer0(p);
+        if (worker < nt0) {
+            w.e = 0;
+            w.n = worker;
+        } else if (worker - nt0 < (p.D - 1) * p.NT) {
+            w.e = 1 + (worker - nt0) / p.NT;
+            w.n = (worker - nt0) - (w.e - 1) * p.NT;
         }
     } else if (p.owner == 2) {
         if (worker < p.NT) {
@@ -353,7 +365,7 @@ FT_HD bool walk_next(const Problem& p, TileWalk& w, TileId& tl, long long& tid) 
         tl.axis = 0;
         tl.m = 0;
         tl.n = w.n;
-        tid = cell_lin(p, w.e, w.t, 0) * p.NT + w.n;
+        tid = cell_lin(p, w.e, w.t, 0) * (p.nt0 > p.NT ? p.nt0 : p.NT) + w.n;
         ++w.t;
         return true;
     }

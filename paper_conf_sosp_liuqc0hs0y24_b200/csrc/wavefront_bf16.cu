@@ -222,7 +222,8 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
     const uint32_t full0 = (CG == 2) ? mapa_shared(smem_u32(full), 0) : smem_u32(full);
     int stage = 0;
     uint32_t phase = 0;
-    const int target = flag_target(P);
+    const int target = flag_target(P), target0 = flag_target_layer(P, 0);
+    const long long l0cells = (long long)P.L0 * P.L1;  // cells of layer 0 come first (cell_lin)
     const int kchunks = P.H / BK;
     uint64_t pol_stream = policy_evict_first();
     uint64_t pol_keep = policy_evict_last();
@@ -256,7 +257,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
                 // that are ready (x, the layer below) stream in while a later producer finishes
                 if (kc == 0 && sg.scell >= 0 && !FT_DEV_BIT(P.debug, 1)) {
                     FT_TR_BEGIN();
-                    wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, target);
+                    wait_flag_geq(T.flags + (long long)sg.scell * P.MB + tl.m, sg.scell < l0cells ? target0 : target);
                     FT_TR_END(TR_P_FLAG);
                     if (rank == 0) FT_EV(tile, 5);
                     fence_proxy_async_global();
@@ -513,9 +514,10 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
     // owner-computes (TileWalk): this thread's rows x units of the slab are the same in every
     // tile, so the cell state stays in registers (cst) from step t to t + 1 — no c ring, no
     // c-ready counter.  Otherwise, under layer bands h and c are published separately ((2b)).
-    const int worker = (int)(blockIdx.x / CG);
+    const int worker = (int)(blockIdx.x / CG), nt0 = nt_layer0(P);
     const bool own = P.owner == 1 || (P.owner == 2 && worker < P.NT) ||
-                     (P.owner == 3 && worker < P.D * P.NT && P.dil[worker / P.NT] == 1);
+                     (P.owner == 3 && (worker < nt0 || (worker - nt0 < (P.D - 1) * P.NT &&
+                                                        P.dil[1 + (worker - nt0) / P.NT] == 1)));
     const bool split = P.band > 0 && !own;
     float cst[EPI_UNITS];
 #pragma unroll
@@ -785,9 +787,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
 }
 
 template <int CG, int U>
-__global__ void __launch_bounds__(THREADS, 1)
-wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
-                      const __grid_constant__ Maps M) {
+__device__ __forceinline__ void kernel_body(const Problem& P, const Tensors& T, const Maps& M) {
     using C = KCfg<CG, U>;
     extern __shared__ uint8_t smem_raw[];
     const uint32_t pad = (1024u - (smem_u32(smem_raw) & 1023u)) & 1023u;
@@ -849,6 +849,24 @@ wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__
     }
     if (threadIdx.x == 0) FT_TR_END(TR_TOTAL);
     FT_TR_FLUSH(threadIdx.x == 0);
+}
+
+// U0 < U: under owner mode 3 the workers of layer 0 (the only recurrence without slack in a
+// dilated nest) run slabs of U0 units — half the MMAs and half the gate math per step on the
+// critical chain, and all of a step's recurrent K chunks fit in the deeper ring of the narrower
+// stage — with their own tensor maps M0; every other worker runs U-unit slabs.  A CTA's role and
+// shared-memory layout are fixed for the whole launch, so each runs one body.
+template <int CG, int U, int U0>
+__global__ void __launch_bounds__(THREADS, 1)
+wavefront_bf16_kernel(const __grid_constant__ Problem P, const __grid_constant__ Tensors T,
+                      const __grid_constant__ Maps M, const __grid_constant__ Maps M0) {
+    if constexpr (U0 != U) {
+        if (P.owner == 3 && (int)(blockIdx.x / CG) < P.nt0) {
+            kernel_body<CG, U0>(P, T, M0);
+            return;
+        }
+    }
+    kernel_body<CG, U>(P, T, M);
 }
 
 // ------------------------------------------------------------------------------ host side
@@ -1071,7 +1089,7 @@ cudaError_t encode_maps(const Problem& p, const Tensors& t, EncodeTiledFn enc, b
 
 template <int CG, int U>
 cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, std::string* err,
-                           const Maps& M, bool x_direct, int dev, int nsm, int* clusters) {
+                           const Maps& M, const Maps* M0, bool x_direct, int dev, int nsm, int* clusters) {
     using C = KCfg<CG, U>;
     cudaError_t e = cudaSuccess;
     const int Bp = p.MB * p.BM;
@@ -1115,7 +1133,7 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
         cfg.numAttrs = 1;
         int nclusters = clusters[dev];
         if (nclusters < 1) {
-            e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U>, &cfg);
+            e = cudaOccupancyMaxActiveClusters(&nclusters, wavefront_bf16_kernel<CG, U, U>, &cfg);
             if (e != cudaSuccess || nclusters < 1) {
                 if (err) *err = std::string("cluster occupancy query: ") + cudaGetErrorString(e);
                 return e != cudaSuccess ? e : cudaErrorInvalidConfiguration;
@@ -1159,6 +1177,14 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
         // profiles/rnd2_ab_owner_all.txt); FT_OWNER_ALL=0 keeps mode 2
         const char* ea = getenv("FT_OWNER_ALL");
         if (q.owner == 2 && !(ea && ea[0] == '0') && (long long)p.D * p.NT <= grid / CG) q.owner = 3;
+        // ... and layer 0 in half-width slabs (wavefront_bf16_kernel<2, 64, 32>) when those fit
+        // too; FT_NARROW0=0 keeps layer 0 at the common width
+        if constexpr (CG == 2 && U == 64) {
+            const char* en = getenv("FT_NARROW0");
+            const int nt0 = p.H / 32;
+            if (q.owner == 3 && M0 && !(en && en[0] == '0') && nt0 + (long long)(p.D - 1) * p.NT <= grid / CG)
+                q.nt0 = nt0;
+        }
     }
     // recurrent half first for dilated layers (segments); FT_REC_FIRST=0 keeps the input half first
     {
@@ -1212,18 +1238,38 @@ cudaError_t launch_cg_maps(const Problem& p, const Tensors& t, cudaStream_t s, s
         *t.ysig_per_step = (t.ysig && q.kind == KIND_SEQ && q.cell == CELL_LSTM)
                                ? q.naxes * q.MB * q.NT * CG * EPI_WARPS : 0;
         if (t.ysig_per_chunk) *t.ysig_per_chunk = q.owner == 1;  // owner walk: once per chunk
+        if (t.nsig0_per_step)  // layer 0's final-state count when it runs narrower slabs
+            *t.nsig0_per_step = (*t.ysig_per_step && q.nt0 > 0) ? q.naxes * q.MB * q.nt0 * CG * EPI_WARPS : 0;
+    }
+    auto kern = wavefront_bf16_kernel<CG, U, U>;
+    const Maps* m0 = &M;
+    if constexpr (CG == 2 && U == 64) {
+        if (q.nt0 > 0) {
+            kern = wavefront_bf16_kernel<2, 64, 32>;
+            m0 = M0;
+            static bool set_mixed[64] = {};
+            if (!set_mixed[dev]) {
+                e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM_BYTES);
+                if (e != cudaSuccess) {
+                    if (err) *err = std::string("bf16 launch setup (narrow layer 0): ") + cudaGetErrorString(e);
+                    return e;
+                }
+                set_mixed[dev] = true;
+            }
+        }
     }
     int coop = 1;
     if constexpr (CG == 2)
-        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, &coop, wavefront_bf16_kernel<CG, U>,
-                                      q, t, M);
+        e = launch_cluster_persistent(cfg, nattr == 2 ? attr2 : attr, nattr, &coop, kern, q, t, M, *m0);
     else
-        e = cudaLaunchKernelEx(&cfg, wavefront_bf16_kernel<CG, U>, q, t, M);
+        e = cudaLaunchKernelEx(&cfg, kern, q, t, M, *m0);
     if (e == cudaSuccess)
         set_last_launch("wavefront_bf16_kernel<" + std::to_string(CG) + "," + std::to_string(U) +
+                        (q.nt0 > 0 ? ",32" : "") +
                         "> grid=" + std::to_string(grid) + " cluster=" + std::to_string(CG) +
                         " cooperative=" + std::to_string(coop) + " band=" + std::to_string(q.band) +
                         " skew=" + std::to_string(seq_skew(q)) + " owner=" + std::to_string(q.owner) +
+                        " nt0=" + std::to_string(nt_layer0(q)) +
                         " x_direct=" + std::to_string(q.x_direct) + " persist_layers=" +
                         std::to_string(q.persist_layers) + " resident_layers=" +
                         std::to_string(q.resident_layers) + " stress=" + std::to_string((q.debug & 64) != 0));
@@ -1259,7 +1305,7 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
     static bool attr_set[64] = {};
     static int clusters[64] = {};
     if (!attr_set[dev]) {
-        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        e = cudaFuncSetAttribute(wavefront_bf16_kernel<CG, U, U>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  C::SMEM_BYTES);
         if (e != cudaSuccess) {
             if (err) *err = std::string("bf16 launch setup: ") + cudaGetErrorString(e);
@@ -1267,7 +1313,24 @@ cudaError_t launch_cg(const Problem& p, const Tensors& t, cudaStream_t s, std::s
         }
         attr_set[dev] = true;
     }
-    return launch_cg_maps<CG, U>(p, t, s, err, M, x_direct, dev, nsm, clusters);
+    // narrow layer-0 slabs (owner mode 3 of a dilated nest): tensor maps of the 32-unit tile
+    Maps M0;
+    const Maps* m0 = nullptr;
+    if constexpr (CG == 2 && U == 64) {
+        bool dilated = false;
+        for (int d = 1; d < p.D; ++d) dilated = dilated || p.dil[d] > 1;
+        if (dilated && p.kind == KIND_SEQ && p.cell == CELL_LSTM && p.dil[0] == 1 && p.H % 64 == 0) {
+            MapsKey k0 = key;
+            k0.units = 32;
+            if (!maps_cache().find(k0, &M0)) {
+                const cudaError_t ee = encode_maps<2, 32>(p, t, enc, x_direct, &M0, err);
+                if (ee != cudaSuccess) return ee;
+                maps_cache().put(k0, M0);
+            }
+            m0 = &M0;
+        }
+    }
+    return launch_cg_maps<CG, U>(p, t, s, err, M, m0, x_direct, dev, nsm, clusters);
 }
 
 }  // namespace

@@ -695,6 +695,29 @@ def test_bf16_all_layers_owner_walk(dil, monkeypatch):
         assert torch.equal(got[k], ref_gpu[k]), k
 
 
+@pytest.mark.parametrize("dil,T", [([1, 2, 4], 9), ([1, 2, 4, 8, 16, 32], 12), ([1, 3, 2], 7)])
+def test_bf16_narrow_layer0_owners(dil, T, monkeypatch):
+    """Owner mode 3 with layer 0 in 32-unit slabs (wavefront_bf16_kernel<2,64,32>, the default
+    for dilated nests when the slabs fit): sampled rows against the oracle (with h_all / c_all),
+    and against the uniform-width walk (FT_NARROW0=0) — every element is the same K-ordered sum,
+    only the N extent of layer 0's MMAs differs — to within one bf16 rounding of h."""
+    monkeypatch.setenv("FT_RESIDENT", "0")
+    B, H, D = 256, 512, len(dil)
+    p = ftgen.stacked_inputs(B, T, H, D, 2040 + D + T, "bf16")
+    got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    assert "wavefront_bf16_kernel<2,64,32>" in ft.ft_last_launch() and "owner=3 nt0=16" in ft.ft_last_launch(), \
+        ft.ft_last_launch()
+    monkeypatch.setenv("FT_NARROW0", "0")
+    uni = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
+    assert "owner=3 nt0=8" in ft.ft_last_launch(), ft.ft_last_launch()
+    rows = [0, 1, 77, 128, 200, 255]
+    _check(got, _oracle_stacked(p, dil=dil, want_all=True, rows=rows), torch.bfloat16, ALL, rows=rows,
+           ctx=f"narrow layer 0 {dil}")
+    for k in ALL:
+        d = normrel(host(got[k]), host(uni[k]))
+        assert d <= 4e-3, f"narrow vs uniform {k}: {d:.3e}"
+
+
 @pytest.mark.parametrize("B,Lx,Ly,H,D,band", [(130, 4, 5, 128, 3, 1), (100, 3, 3, 64, 4, 2), (256, 2, 6, 128, 2, 1)])
 def test_bf16_grid_depth_bands(B, Lx, Ly, H, D, band, monkeypatch):
     """Grid RNN in depth bands (FT_BAND): parity with the oracle and bitwise equality with the

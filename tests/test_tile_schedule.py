@@ -307,6 +307,43 @@ def test_all_layers_owner_walk(D, T, nt, nw, dil):
     assert ft.ft_tile_walk(D, T, 0, 1, 3, nt, 0, D * nt - 1) == ft.ft_tile_walk(D, T, 0, 1, 0, nt, 0, D * nt - 1)
 
 
+@pytest.mark.parametrize("D,T,nt,nw,dil", [
+    (6, 12, 8, 74, [1, 2, 4, 8, 16, 32]), (3, 7, 4, 17, [1, 3, 2]), (4, 5, 2, 11, [1, 1, 2, 1]),
+])
+def test_all_layers_owner_walk_narrow_layer0(D, T, nt, nw, dil):
+    """Owner mode 3 with layer 0 in half-width slabs (owner code 4): workers < 2·nt own layer 0's
+    half-width N-tiles, the next (D-1)·nt the other layers' slabs.  Every layer-0 half tile and
+    every other (d, t, n) exactly once; deadlock-free when a cell completes after all of its
+    tiles (2·nt on layer 0)."""
+    walks = [ft.ft_tile_walk(D, T, 0, 1, 4, nt, w, nw) for w in range(nw)]
+    allt = sorted(x for w in walks for x in w)
+    want = sorted([(0, t, n) for t in range(T) for n in range(2 * nt)] +
+                  [(d, t, n) for d in range(1, D) for t in range(T) for n in range(nt)])
+    assert allt == want
+    for w in range(nw):
+        if w < 2 * nt:
+            assert walks[w] == [(0, t, w) for t in range(T)]
+        elif w < 2 * nt + (D - 1) * nt:
+            e, n = 1 + (w - 2 * nt) // nt, (w - 2 * nt) % nt
+            assert walks[w] == [(e, t, n) for t in range(T)]
+        else:
+            assert walks[w] == []
+    left = {(d, t): (2 * nt if d == 0 else nt) for d in range(D) for t in range(T)}
+    heads = [0] * nw
+    while any(heads[w] < len(walks[w]) for w in range(nw)):
+        done = []
+        for w in range(nw):
+            if heads[w] < len(walks[w]):
+                d, t, n = walks[w][heads[w]]
+                if (d == 0 or left[(d - 1, t)] == 0) and (t < dil[d] or left[(d, t - dil[d])] == 0):
+                    done.append(w)
+        assert done, "deadlock"
+        for w in done:
+            d, t, n = walks[w][heads[w]]
+            heads[w] += 1
+            left[(d, t)] -= 1
+
+
 @pytest.mark.parametrize("D,Lx,Ly,band", [(4, 3, 4, 1), (4, 5, 2, 2), (5, 4, 4, 3), (3, 1, 6, 1), (2, 6, 1, 1)])
 def test_grid_depth_bands_are_legal(D, Lx, Ly, band):
     """Grid nests in depth bands (band after band, each a wavefront over i + j + (d - d0)): every
