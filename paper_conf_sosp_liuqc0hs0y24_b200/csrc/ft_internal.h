@@ -56,7 +56,8 @@ struct Tensors {
     // every epilogue warp fences at system scope and adds 1 to nsig[d]; a second copy stream
     // moves layer d's rows to the host once nsig[d] reaches *ysig_per_step (same count per cell)
     int* nsig = nullptr;
-    int* nsig0_per_step = nullptr; // HOST: nsig[0]'s count when layer 0 runs narrower slabs
+    int* nsig0_per_step = nullptr; // HOST: nsig[0]'s count when layer 0 runs narrower slabs (dilated
+                                   // nests only; the host-buffer call takes stacked nests)
                                    // (owner mode 3); 0 = *ysig_per_step
     int* ysig_per_chunk = nullptr; // HOST: 1 = owner walk: each warp signals once per chunk (its
                                    // last step of the chunk), so a chunk completes at per_step

@@ -627,6 +627,7 @@ def test_bf16_layer_bands_stress(monkeypatch):
     (100, 10, 128, 3, {"FT_RESIDENT": "0"}),                                   # 1-CTA tiles, T = chunk
     (64, 9, 256, 8, {}),                                                       # cluster/resident: no signal
     (256, 12, 128, 4, {"FT_RESIDENT": "0", "FT_OWNER_L0": "1"}),               # layer-0 owners: per-tile y signals
+    (256, 9, 512, 3, {"FT_RESIDENT": "0", "FT_OWNER_L0": "1"}),                # every layer owned (mode 3)
 ])
 def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
     """ft_stacked_lstm_fwd_hostio (pinned host in/out; y copied to the host in time chunks while
@@ -646,6 +647,8 @@ def test_bf16_hostio_matches_device_path(B, T, H, D, env, monkeypatch):
     nb = ft.ft_stacked_lstm_hostio_workspace_size(B, T, H, D, ft.FT_BF16)
     ws = torch.empty(nb, dtype=torch.uint8, device="cuda")
     s = torch.cuda.Stream()
+    if H == 512:
+        assert "owner=3" in ft.ft_last_launch(), ft.ft_last_launch()
     for _ in range(2):  # twice: the per-chunk counters are reset by every call
         ft.check(ft.ft_stacked_lstm_fwd_hostio(B, T, H, D, ft.FT_BF16, x_h.data_ptr(), W.data_ptr(),
                                                U.data_ptr(), b.data_ptr(), y_h.data_ptr(), hn_h.data_ptr(),
