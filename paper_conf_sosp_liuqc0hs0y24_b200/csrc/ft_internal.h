@@ -56,9 +56,9 @@ struct Tensors {
     // every epilogue warp fences at system scope and adds 1 to nsig[d]; a second copy stream
     // moves layer d's rows to the host once nsig[d] reaches *ysig_per_step (same count per cell)
     int* nsig = nullptr;
-    int* nsig0_per_step = nullptr; // HOST: nsig[0]'s count when layer 0 runs narrower slabs (dilated
-                                   // nests only; the host-buffer call takes stacked nests)
-                                   // (owner mode 3); 0 = *ysig_per_step
+    int* nsig0_per_step = nullptr; // HOST: nsig[0]'s count when layer 0 runs narrower slabs (owner
+                                   // mode 3 of dilated nests; the host-buffer call itself takes
+                                   // stacked nests); 0 = *ysig_per_step
     int* ysig_per_chunk = nullptr; // HOST: 1 = owner walk: each warp signals once per chunk (its
                                    // last step of the chunk), so a chunk completes at per_step
 };
