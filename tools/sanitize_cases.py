@@ -77,5 +77,7 @@ os.environ["FT_BAND"] = "2"                               # SSA slot rings wrapp
 run_seq(256, 11, 64, 6, torch.bfloat16, resident="0")
 os.environ.pop("FT_BAND")
 run_seq(256, 11, 64, 4, torch.bfloat16, dil=[1, 2, 4, 3], resident="0")  # rings + layer-0 owners (default)
+# last session of round 2: every layer owned (mode 3), 32-unit layer-0 slabs (<2,64,32>), recurrent half first
+run_seq(256, 7, 512, 4, torch.bfloat16, dil=[1, 2, 4, 8], resident="0")
 torch.cuda.synchronize()
 print("sanitize cases done")
