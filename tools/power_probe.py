@@ -24,6 +24,12 @@ def make_fn(mode):
     from paper_conf_sosp_liuqc0hs0y24_b200 import ft
     c = ftgen.CONFIGS[mode]
     ws = ft.Workspace()
+    if c["kind"] == "grid":
+        g = ftgen.grid_inputs(c["batch"], c["len_x"], c["len_y"], c["hidden"], c["depth"], 1, "bf16")
+        a = [torch.from_numpy(g[k]).cuda().to(torch.bfloat16) for k in ("x", "ys", "W", "U")] + \
+            [torch.from_numpy(g["b"]).cuda()]
+        return (lambda: ft.grid_rnn(*a, workspace=ws)), \
+            48 * c["hidden"] ** 2 * c["len_x"] * c["len_y"] * c["depth"] * c["batch"]
     p = ftgen.stacked_inputs(c["batch"], c["seq"], c["hidden"], c["depth"], 1, "bf16")
     a = [torch.from_numpy(p[k]).cuda().to(torch.bfloat16) for k in ("x", "W", "U")] + [torch.from_numpy(p["b"]).cuda()]
     dil = list(c.get("dilations", [])) or None
