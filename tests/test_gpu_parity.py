@@ -702,24 +702,26 @@ def test_bf16_all_layers_owner_walk(dil, monkeypatch):
         assert torch.equal(got[k], ref_gpu[k]), k
 
 
-@pytest.mark.parametrize("dil,T", [([1, 2, 4], 9), ([1, 2, 4, 8, 16, 32], 12), ([1, 3, 2], 7)])
-def test_bf16_narrow_layer0_owners(dil, T, monkeypatch):
+@pytest.mark.parametrize("dil,T,B,H", [([1, 2, 4], 9, 256, 512), ([1, 2, 4, 8, 16, 32], 12, 256, 512),
+                                       ([1, 3, 2], 7, 256, 512), ([1, 2, 4, 8], 13, 200, 384),
+                                       ([1, 5, 2], 6, 256, 1024)])
+def test_bf16_narrow_layer0_owners(dil, T, B, H, monkeypatch):
     """Owner mode 3 with layer 0 in 32-unit slabs (wavefront_bf16_kernel<2,64,32>, the default
     for dilated nests when the slabs fit): sampled rows against the oracle (with h_all / c_all),
     and against the uniform-width walk (FT_NARROW0=0) — every element is the same K-ordered sum,
     only the N extent of layer 0's MMAs differs — to within one bf16 rounding of h."""
     monkeypatch.setenv("FT_RESIDENT", "0")
-    B, H, D = 256, 512, len(dil)
+    D = len(dil)
     p = ftgen.stacked_inputs(B, T, H, D, 2040 + D + T, "bf16")
     got = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
-    assert "wavefront_bf16_kernel<2,64,32>" in ft.ft_last_launch() and "owner=3 nt0=16" in ft.ft_last_launch(), \
-        ft.ft_last_launch()
+    assert "wavefront_bf16_kernel<2,64,32>" in ft.ft_last_launch() and f"owner=3 nt0={H // 32}" in \
+        ft.ft_last_launch(), ft.ft_last_launch()
     monkeypatch.setenv("FT_NARROW0", "0")
     uni = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
-    assert "owner=3 nt0=8" in ft.ft_last_launch(), ft.ft_last_launch()
-    rows = [0, 1, 77, 128, 200, 255]
+    assert f"owner=3 nt0={H // 64}" in ft.ft_last_launch(), ft.ft_last_launch()
+    rows = [0, 1, 77, 128, B - 56, B - 1]
     _check(got, _oracle_stacked(p, dil=dil, want_all=True, rows=rows), torch.bfloat16, ALL, rows=rows,
-           ctx=f"narrow layer 0 {dil}")
+           ctx=f"narrow layer 0 {dil} B={B} H={H}")
     for k in ALL:
         d = normrel(host(got[k]), host(uni[k]))
         assert d <= 4e-3, f"narrow vs uniform {k}: {d:.3e}"
