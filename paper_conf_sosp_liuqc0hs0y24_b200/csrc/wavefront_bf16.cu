@@ -91,7 +91,15 @@ __device__ unsigned long long g_events[EV_MAX_TILES * EV_K];
 #define FT_TR_END(slot) ((void)0)
 #define FT_TR_ADD(slot, v) ((void)0)
 #define FT_TR_FLUSH(cond) ((void)0)
+#ifdef FT_TRACE_LIGHT  // development (tools/c4_spread.py): events 1-5, 7-11 only, no role
+                       // counters — close to the release build's timing
+constexpr int EV_MAX_TILES = 32768;
+constexpr int EV_K = 16;
+__device__ unsigned long long g_events[EV_MAX_TILES * EV_K];
+#define FT_EV(tile, k) do { if ((k) != 0 && (k) != 6 && (k) != 12 && (tile) < EV_MAX_TILES) g_events[(tile) * EV_K + (k)] = globaltimer_ns(); } while (0)
+#else
 #define FT_EV(tile, k) ((void)0)
+#endif
 #endif
 
 namespace {
@@ -271,7 +279,7 @@ __device__ __forceinline__ void run_producer(const Problem& P, const Tensors& T,
             if constexpr (kWeights) FT_TR_BEGIN();
             mbar_wait(&empty[stage], phase ^ 1);
             if constexpr (kWeights) FT_TR_END(TR_P_EMPTY);
-#ifdef FT_TRACE
+#if defined(FT_TRACE) || defined(FT_TRACE_LIGHT)
             if constexpr (!kWeights) {
                 if (rank == 0 && c == nchunks - kchunks) FT_EV(tile, 8);
                 if (rank == 0 && c == nchunks - 1) FT_EV(tile, 9);
@@ -338,7 +346,7 @@ __device__ __forceinline__ void run_mma(const Problem& P, uint32_t tmem_base, ui
             FT_TR_BEGIN();
             mbar_wait_warp(&full[stage], phase);
             FT_TR_END(TR_M_FULL);
-#ifdef FT_TRACE
+#if defined(FT_TRACE) || defined(FT_TRACE_LIGHT)
             if ((threadIdx.x & 31) == 0 && c == nchunks - kchunks) FT_EV(tile, 10);
             if ((threadIdx.x & 31) == 0 && c == nchunks - kchunks - 1) FT_EV(tile, 11);
 #endif
@@ -1347,6 +1355,8 @@ extern "C" __attribute__((visibility("default"))) int ft_debug_trace(unsigned lo
     }
     return TR_SLOTS;
 }
+#endif
+#if defined(FT_TRACE) || defined(FT_TRACE_LIGHT)
 extern "C" __attribute__((visibility("default"))) int ft_debug_events(unsigned long long* host, int ntiles) {
     if (ntiles > EV_MAX_TILES) ntiles = EV_MAX_TILES;
     cudaDeviceSynchronize();
