@@ -52,7 +52,8 @@ print("tiles by median release lag:", [(int(k), round(float(np.nanmedian(R[:, k]
 names = {5: "A producer saw the flag", 8: "A producer got the slot of the first recurrent chunk",
          11: "MMA warp saw the last input-half chunk land", 9: "A producer got the slot of the last chunk", 2: "A loads issued",
          10: "MMA warp saw the first recurrent chunk land", 7: "MMA warp issued the last chunk",
-         3: "epilogue saw the accumulator", 4: "released"}
-for k in (11, 5, 8, 9, 2, 10, 7, 3, 4):
+         3: "epilogue saw the accumulator", 13: "epilogue: first TMEM chunk in registers",
+         14: "epilogue: math and h stores issued (leader warp)", 4: "released"}
+for k in (11, 5, 8, 9, 2, 10, 7, 3, 13, 14, 4):
     v = np.nanmax(ev[0, 1:, :nt0, k], 1) - np.nanmax(R[:-1], 1)
     print(f"  +{np.nanmedian(v):5.2f} us  {names[k]}")
