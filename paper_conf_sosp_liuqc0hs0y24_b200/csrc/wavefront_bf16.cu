@@ -97,6 +97,7 @@ constexpr int EV_MAX_TILES = 32768;
 constexpr int EV_K = 16;
 __device__ unsigned long long g_events[EV_MAX_TILES * EV_K];
 #define FT_EV(tile, k) do { if ((k) != 0 && (k) != 6 && (k) != 12 && (tile) < EV_MAX_TILES) g_events[(tile) * EV_K + (k)] = globaltimer_ns(); } while (0)
+// (13 first TMEM chunk in the epilogue's registers, 14 math and h stores issued: light build only)
 #else
 #define FT_EV(tile, k) ((void)0)
 #endif
@@ -620,6 +621,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
             tmem_ld_32x32b<CH>(tbase + 2 * U + u0, zo);
             tmem_ld_32x32b<CH>(tbase + 3 * U + u0, zg);
             tmem_wait_ld();
+            if (u0 == 0 && leader_thread && rank == 0) FT_EV(tile, 13);  // first TMEM chunk in registers
 #ifdef FT_TRACE
             if (leader_thread) _acc[TR_E_LDTM] += clock64() - _e0;
             _e0 = clock64();
@@ -702,6 +704,7 @@ __device__ __forceinline__ void run_epilogue(const Problem& P, const Tensors& T,
         if (leader_thread) _acc[TR_E_STORE] += clock64() - _e1;
         _e1 = clock64();
 #endif
+        if (leader_thread && rank == 0) FT_EV(tile, 14);  // math and h stores issued (light trace)
         __syncwarp();  // orders the warp's stores before lane 0's release (bar.warp.sync)
 #ifdef FT_TRACE
         if (leader_thread) _acc[TR_E_BAR] += clock64() - _e1;
