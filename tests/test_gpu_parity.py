@@ -444,6 +444,37 @@ def test_bf16_cuda_graph_capture_replay(band, shape, monkeypatch):
     _check(out, ref, torch.bfloat16, OUT, ctx=f"graph band={band}")
 
 
+def test_bf16_cuda_graph_dilated_mixed_kernel():
+    """C4's schedule (every layer owned, 32-unit layer-0 slabs in the same launch as the 64-unit
+    upper layers) captured into a CUDA graph and replayed twice with new inputs: both replays
+    match the oracle on sampled rows."""
+    B, T, H, dil = 256, 7, 384, [1, 2, 4, 8]
+    D = len(dil)
+    p1 = ftgen.stacked_inputs(B, T, H, D, 1828, "bf16")
+    x, W, U = (dev(p1[k], torch.bfloat16) for k in ("x", "W", "U"))
+    b = dev(p1["b"], torch.float32)
+    ws = ft.Workspace()
+    s = torch.cuda.Stream()
+    out = {"y": torch.empty((B, T, H), dtype=torch.bfloat16, device="cuda"),
+           "h_n": torch.empty((B, D, H), dtype=torch.bfloat16, device="cuda"),
+           "c_n": torch.empty((B, D, H), dtype=torch.float32, device="cuda")}
+    with torch.cuda.stream(s):
+        ft.dilated_rnn(x, W, U, b, dil, workspace=ws, out=out, stream=s)
+    s.synchronize()
+    assert "wavefront_bf16_kernel<2,64,32>" in ft.ft_last_launch(), ft.ft_last_launch()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        ft.dilated_rnn(x, W, U, b, dil, workspace=ws, out=out, stream=s)
+    rows = [0, 100, 255]
+    for seed in (1829, 1830):
+        p2 = ftgen.stacked_inputs(B, T, H, D, seed, "bf16")
+        x.copy_(dev(p2["x"], torch.bfloat16))
+        g.replay()
+        torch.cuda.synchronize()
+        ref = oracle.dilated_rnn(p2["x"][rows], p1["W"], p1["U"], p1["b"], dil)
+        _check(out, ref, torch.bfloat16, OUT, rows=rows, ctx=f"graph dilated mixed seed={seed}")
+
+
 # ------------------------------------------------------------------------- NEXT-4: B2B GEMMs
 @pytest.mark.parametrize("M,N", [(128, 128), (256, 512), (1024, 4096), (384, 128)])
 def test_bf16_b2b_gemm(M, N):
