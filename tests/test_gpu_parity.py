@@ -713,15 +713,16 @@ def test_bf16_layer0_owner_walk(dil, monkeypatch):
         assert torch.equal(got[k], ref_gpu[k]), k
 
 
+@pytest.mark.parametrize("B", [256, 100])  # CTA-pair tiles; 1-CTA tiles (B <= 128)
 @pytest.mark.parametrize("dil", [[1, 2, 4, 8, 16, 32], [1, 3, 2], [1, 1, 2, 1]])
-def test_bf16_all_layers_owner_walk(dil, monkeypatch):
+def test_bf16_all_layers_owner_walk(dil, B, monkeypatch):
     """Every layer owned (TileWalk mode 3, the default for dilated nests when D·NT slabs fit):
     parity with the oracle and bitwise equality with the layer-0 owner walk (FT_OWNER_ALL=0: the
     same tiles and K order, another assignment); dilation-1 layers above layer 0 keep c in
     registers, the others use the c ring."""
     monkeypatch.setenv("FT_RESIDENT", "0")
     D = len(dil)
-    p = ftgen.stacked_inputs(256, 9, 128, D, 2030 + D, "bf16")
+    p = ftgen.stacked_inputs(B, 9, 128, D, 2030 + D, "bf16")
     monkeypatch.setenv("FT_OWNER_ALL", "0")
     ref_gpu = _run_stacked(p, torch.bfloat16, dil=dil, want_all=True)
     assert "owner=2" in ft.ft_last_launch()
