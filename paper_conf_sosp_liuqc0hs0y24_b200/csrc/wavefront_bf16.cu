@@ -18,6 +18,10 @@
 //           128 A rows and HALF of the N = 256 weight columns (gates i,f or o,ĝ); the leader CTA
 //           issues M256 N256 K16 MMAs reading both CTAs' shared memory, so each weight tile is
 //           fetched once per cell for the whole 256-row batch and per-CTA weight traffic halves.
+// Each comes in 64-unit (N = 256) and 32-unit (N = 128) N-tiles.  Dilated nests run one launch
+// with two widths (wavefront_bf16_kernel<2, 64, 32>): the CTA pairs that own layer 0 — the only
+// recurrence without slack — run 32-unit slabs, every other pair 64-unit slabs (kernel_body per
+// CTA; TileWalk owner mode 3 in ft_common.cuh).
 //
 // Warp roles (352 threads per CTA with the default FT_EPI_WARPS = 8; 16 epilogue warps measured
 // slower: C3 6.30 -> 6.61 ms, C4 0.871 -> 0.903 ms, profiles/r2_ab_epi_warps.txt):
